@@ -1,0 +1,348 @@
+#!/usr/bin/env python
+"""LowDiff hot-path benchmark (BASELINE.json metric: "diff-build & replay gradient GB/s at
+1/2/4/8 B200, % of HBM roofline").
+
+One STEP = one pass of the whole hot path over one batch:
+  for each of the B iterations of the batch: compress (top-k + EF) -> sparse all-gather (NCCL for
+  P > 1) + coalesce of this rank's shard -> ring slot;
+  then batch merge of the B differentials (STACK, Adam) -> record -> async D2H stage into pinned
+  host memory (copy stream) -> replay of the record onto this rank's full-checkpoint shard.
+value = gradient bytes all ranks fed through the path per second = P * B * n * sizeof(g) / t_step.
+
+Workload (N = 1 line): config C3 = BASELINE configs[2], the VGG-16-shaped gradient the metric's
+1/2/4/8-GPU scaling is quoted on (n = 138,357,544 fp32, rho = 0.001, B = 16, Adam replay of the
+batch's 16 iterations). Inputs are synthetic (workloads/, seeded), resident in HBM before timing;
+every gradient (553 MB) is larger than the 126 MB L2, so no flush is needed between steps.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config 3] [--impl ours|reference]
+  torchrun --nproc-per-node N bench.py --gpus N ...
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+REASONS = {  # nvidia-smi clocks_event_reasons bits
+    0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+    0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+    0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+
+def parse_args():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--profile-steps", type=int, default=-1,
+                    help="steps whose kernels are bracketed by CUDA events (-1: all timed steps)")
+    return ap.parse_args()
+
+
+# ---------------------------------------------------------------------------------------------
+# CPU oracle arm (cpu_baseline and --impl reference): the oracle as it stands, bounded sample
+# ---------------------------------------------------------------------------------------------
+def oracle_step_sample(cfg, n_s: int, t0: int = 0):
+    """Time the oracle on one step of the same workload restricted to the first n_s gradient
+    elements (same rho, B, optimizer): B compress + coalesce, one merge, one replay. Returns
+    (seconds, gradient bytes processed)."""
+    import numpy as np
+    import oracle
+    from workloads import gradient, segment_sigmas
+    sig = segment_sigmas(cfg)[:n_s]
+    k = max(1, int(cfg.rho * n_s))
+    grads = [gradient(cfg, 0, t0 + t, "cpu", sigmas=sig, n=n_s) for t in range(cfg.B)]
+    grads = [g.view(np.int16).numpy().view(np.uint16) if cfg.gdt == "bf16" else g.numpy() for g in
+             [gg.view(__import__("torch").int16) if cfg.gdt == "bf16" else gg for gg in grads]]
+    r = np.zeros(n_s, np.float32)
+    lr = np.float32(cfg.hyper["lr"])
+    x = np.zeros(n_s, np.float32); m = np.zeros(n_s, np.float32); v = np.zeros(n_s, np.float32)
+    o_vdt = oracle.BF16 if cfg.vdt == "bf16" else oracle.F32
+    t_start = time.perf_counter()
+    diffs = []
+    for t in range(cfg.B):
+        idx, val, r = oracle.compress(grads[t], r, k, o_vdt)
+        diffs.append(oracle.coalesce([oracle.pairs_pack(idx, val, o_vdt)], k, o_vdt, 0, n_s, True))
+    mode = oracle.STACK if cfg.merge == "stack" else oracle.SUM
+    rec = oracle.batch_merge(diffs, lr, mode, n_s, 0, n_s, t0, 1)
+    st = {"x": x, "m": m if cfg.opt != "sgd" else None, "v": v if cfg.opt == "adam" else None,
+          "n": n_s, "lo": 0, "hi": n_s, "t": t0, "adam_step": 1000, "momentum_initialized": 1}
+    opt = {"kind": cfg.opt, **{k2: v2 for k2, v2 in cfg.hyper.items() if k2 != "lr"}}
+    oracle.replay(opt, st, [rec])
+    dt = time.perf_counter() - t_start
+    gbytes = cfg.B * n_s * (2 if cfg.gdt == "bf16" else 4)
+    return dt, gbytes
+
+
+def run_reference(args, cfg):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return  # rank 0 alone runs the CPU oracle arm
+    n_s = max(1 << 16, cfg.n // 64)
+    for w in range(args.warmup):
+        oracle_step_sample(cfg, n_s, t0=0)
+    times, gb = [], 0
+    for s in range(args.steps):
+        dt, gb = oracle_step_sample(cfg, n_s, t0=0)
+        times.append(dt)
+    tot = sum(times)
+    val = args.steps * gb / tot / 1e9
+    sample = (f"oracle (plain C++, 1 thread) full step of {cfg.name} on the first {n_s} of n={cfg.n} "
+              f"gradient elements (rho={cfg.rho}, B={cfg.B}, {cfg.opt} replay)")
+    line = {"impl": "reference", "metric": "diff-build & replay gradient GB/s at 1/2/4/8 B200, % of HBM roofline",
+            "value": val, "unit": "GB/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * tot / args.steps, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f32" if cfg.gdt == "f32" else "bf16", "data": "synthetic",
+            "config": {"workload": cfg.name, "n": cfg.n, "n_sample": n_s, "rho": cfg.rho, "B": cfg.B,
+                       "replay": cfg.opt},
+            "cpu_baseline": {"value": val, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": val, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------------------------------------
+# GPU arm
+# ---------------------------------------------------------------------------------------------
+class ClockSampler:
+    def __init__(self, index: int):
+        self.index, self.proc, self.path = index, None, None
+
+    def start(self):
+        try:
+            self.path = os.path.join("/tmp", f"lowdiff_clocks_{os.getpid()}.csv")
+            self.f = open(self.path, "w")
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index),
+                 "--query-gpu=clocks.sm,clocks.max.sm,clocks_event_reasons.active",
+                 "--format=csv,noheader,nounits", "-lms", "100"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.f.close()
+        sm, mx, reasons = [], 0.0, set()
+        for line in open(self.path):
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) < 3:
+                continue
+            try:
+                sm.append(float(parts[0])); mx = max(mx, float(parts[1]))
+                bits = int(parts[2], 16)
+                for b, name in REASONS.items():
+                    if bits & b and name != "gpu_idle":
+                        reasons.add(name)
+            except ValueError:
+                continue
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def run_ours(args, cfg):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sc_yaolhlzz25_b200 as ld
+    from paper_conf_sc_yaolhlzz25_b200 import build
+    from workloads import full_checkpoint, gradient, segment_sigmas
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    assert world == args.gpus or world == 1, "--gpus must match the torchrun world size"
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    build.build()
+    P = world
+    n, k, B = cfg.n, cfg.k, cfg.B
+    gsz = 2 if cfg.gdt == "bf16" else 4
+    lo, hi = ld.shard_bounds(n, P, rank)
+    comm = ld.Comm(P, rank) if P > 1 else None
+
+    # ---- resident inputs: B gradients (seeded, per rank), residual, full-checkpoint shard ----
+    sig = segment_sigmas(cfg, dev)
+    grads = [gradient(cfg, rank, t, dev, sigmas=sig) for t in range(B)]
+    del sig
+    r = torch.zeros(n, device=dev)
+    ck = full_checkpoint(cfg, lo, hi, dev)
+    state = {"x": ck["x"], "m": ck["m"], "v": ck["v"], "x_bf16": None, "n": n, "lo": lo, "hi": hi,
+             "t": 0, "adam_step": ck["adam_step"], "momentum_initialized": ck["momentum_initialized"]}
+    opt = {"kind": cfg.opt, **{kk: vv for kk, vv in cfg.hyper.items() if kk != "lr"}}
+    lr = float(np.float32(cfg.hyper["lr"]))
+    cap = min(P * k, hi - lo)
+    ring = [(torch.empty(cap, dtype=torch.int32, device=dev), torch.empty(cap, device=dev),
+             torch.zeros(1, dtype=torch.int64, device=dev)) for _ in range(B)]
+    pairs = torch.empty(ld.pairs_bytes(k, cfg.vdt), dtype=torch.uint8, device=dev)
+    rec_cap = ld.record_max_bytes(cfg.merge, B, B * cap)
+    record = torch.empty(rec_cap, dtype=torch.uint8, device=dev)
+    d_bytes = torch.zeros(1, dtype=torch.int64, device=dev)
+    head = torch.empty(80 + 4 * B + 16, dtype=torch.uint8, pin_memory=True)
+    staged = torch.empty(rec_cap, dtype=torch.uint8, pin_memory=True)
+    main = torch.cuda.current_stream()
+    copy_stream = torch.cuda.Stream()
+    t_iter = [0]
+
+    def step(inputs=None, h2d=None):
+        """One pass of the path over one batch; returns staged record bytes."""
+        for j in range(B):
+            if h2d is not None:               # e2e: this iteration's gradient from pinned host memory
+                h2d[0][j % len(h2d[0])].copy_(h2d[1][j % len(h2d[1])], non_blocking=True)
+                g = h2d[0][j % len(h2d[0])]
+            else:
+                g = grads[j]
+            ld.compress(g, r, k, vdt=cfg.vdt, pairs=pairs)
+            ld.allgather_sparse(comm, pairs, k, cfg.vdt, lo, hi, True, *ring[j])
+        diffs = [(ring[j][0], ring[j][1], ring[j][2], cap, lr) for j in range(B)]
+        ld.batch_merge(diffs, cfg.merge, n, lo, hi, t_iter[0], P, record=record, d_record_bytes=d_bytes)
+        nb = ld.record_bytes(d_bytes, rec_cap)          # the checkpoint thread's only sync
+        ld.stage_d2h(record, 80 + 4 * B, head, main)    # header + lr[] for the host-side replay call
+        copy_stream.wait_stream(main)
+        ld.stage_d2h(record, nb, staged, copy_stream)   # async persist staging (copy engine)
+        main.synchronize()
+        state["t"] = t_iter[0]
+        ld.replay(state, opt, [(record, head)])
+        main.wait_stream(copy_stream)
+        t_iter[0] += B
+        return nb
+
+    def timed(nsteps, **kw):
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        nb = 0
+        for _ in range(nsteps):
+            nb = step(**kw)
+        e1.record()
+        torch.cuda.synchronize()
+        ms = e0.elapsed_time(e1)
+        if world > 1:
+            t = torch.tensor([ms], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = float(t.item())
+            dist.barrier()
+        return ms, nb
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    clocks = ClockSampler(local)
+    clocks.start()
+    launches0 = ld.launch_count()
+    ld.profile_enable(True)
+    ms, rec_bytes = timed(args.steps)
+    ld.profile_enable(False)
+    launches = ld.launch_count() - launches0
+    clk = clocks.stop()
+    prof = {c: ld.profile_query(c) for c in ("compress_stream", "compress_sample", "compress_select",
+                                             "compress_emit", "coalesce", "starts", "merge", "merge_pack",
+                                             "replay_dense", "replay_sparse")}
+    ms_step = ms / args.steps
+    value = P * B * n * gsz / (ms_step * 1e-3) / 1e9
+
+    # ---- roofline of the dominant kernel (measured live over the timed region) ----
+    peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
+        os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
+    hbm_peak = float(peaks.get("hbm_gbs", 6650.0))
+    peak_note = "MEASURED_PEAKS.json hbm_gbs (measured copy)" if "hbm_gbs" in peaks else "fallback 6.65 TB/s"
+    cs_ms, cs_n = prof["compress_stream"]
+    alg_bytes = (gsz + 8) * n + (4 + (2 if cfg.vdt == "bf16" else 4) + 4) * k   # read g,r; write r; pairs; r on S
+    achieved = alg_bytes / (cs_ms / cs_n * 1e-3) / 1e9 if cs_n else 0.0
+    traffic = None
+    summ = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if os.path.exists(summ):
+        try:
+            traffic = json.load(open(summ)).get(cfg.name, {}).get("compress_stream", {}).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    total_prof = sum(v[0] for v in prof.values()) or 1.0
+    kernels = {c: {"ms_per_step": v[0] / args.steps, "launches_per_step": v[1] / args.steps,
+                   "share": v[0] / total_prof} for c, v in prof.items() if v[1]}
+    roofline = {"bound": "hbm", "kernel": "compress_stream", "achieved": achieved, "peak": hbm_peak,
+                "unit": "GB/s", "frac": achieved / hbm_peak, "traffic": traffic,
+                "alg_bytes_per_launch": alg_bytes, "launch_ms": cs_ms / cs_n if cs_n else None,
+                "peak_source": peak_note}
+
+    # ---- e2e: same metric through the public API with host buffers (pinned H2D of every gradient) ----
+    e2e = None
+    if not args.no_e2e:
+        npool = min(B, 2)
+        hpool = [torch.empty(n, dtype=grads[0].dtype, pin_memory=True) for _ in range(npool)]
+        for i in range(npool):
+            hpool[i].copy_(grads[i])
+        dpool = [torch.empty_like(grads[0]) for _ in range(npool)]
+        del grads
+        torch.cuda.empty_cache()
+        step(h2d=(dpool, hpool))
+        e_steps = max(1, min(args.steps, 3))
+        ems, enb = timed(e_steps, h2d=(dpool, hpool))
+        e_ms = ems / e_steps
+        e2e = {"value": P * B * n * gsz / (e_ms * 1e-3) / 1e9, "unit": "GB/s",
+               "h2d_bytes_per_step": B * n * gsz, "d2h_bytes_per_step": int(enb) + 80 + 4 * B + 8,
+               "ms_per_step": e_ms, "steps": e_steps}
+
+    # ---- CPU oracle baseline (rank 0, N = 1 only) ----
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        n_s = max(1 << 16, cfg.n // 16)
+        dt, gb = oracle_step_sample(cfg, n_s)
+        cpu = {"value": gb / dt / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
+               "sample": f"one full step of {cfg.name} on the first {n_s} of n={cfg.n} elements "
+                         f"(B={cfg.B} compress+coalesce, merge, {cfg.opt} replay), {dt:.1f} s"}
+
+    if rank == 0:
+        line = {"metric": "diff-build & replay gradient GB/s at 1/2/4/8 B200, % of HBM roofline",
+                "value": value, "unit": "GB/s", "n_gpus": P, "steps": args.steps, "warmup": args.warmup,
+                "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                "dtype": "f32" if cfg.gdt == "f32" else "bf16", "data": "synthetic",
+                "config": {"workload": cfg.name, "n": n, "k": k, "rho": cfg.rho, "B": B, "P": P,
+                           "shard": [lo, hi], "replay": f"{cfg.opt}, {B} iterations (1 {cfg.merge.upper()} record)",
+                           "l2": "inputs larger than L2 (each gradient 553 MB > 126 MB), no flush",
+                           "differentials_per_s": P * B / (ms_step * 1e-3),
+                           "replayed_iterations_per_s": B / (ms_step * 1e-3),
+                           "record_bytes": int(rec_bytes)},
+                "roofline": roofline, "kernels": kernels, "cpu_baseline": cpu, "e2e": e2e,
+                "gpu_launches": int(launches), "clocks": clk}
+        print(json.dumps(line), flush=True)
+    if comm is not None:
+        comm.destroy()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse_args()
+    from workloads import CONFIGS
+    cfg = CONFIGS[args.config]
+    if args.impl == "reference":
+        run_reference(args, cfg)
+    else:
+        run_ours(args, cfg)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,236 @@
+/*
+ * lowdiff.h — C ABI of the B200-native LowDiff hot path (liblowdiff.so).
+ *
+ * LowDiff (Yao et al., SC'25; /root/reference/PAPER.md, cited P:line) reuses each training
+ * iteration's compressed, synchronized gradient G~_t as the differential checkpoint C^D_t
+ * (Finding 1), batches B of them into one write (§4.2) and replays the chain
+ * onto a full checkpoint on recovery (Alg.1 lines 16-24). The five calls below are
+ * the data-parallel hot path BASELINE.json north_star names:
+ *
+ *   lowdiff_compress          Comp(G_{i,t})        Alg.1 line 4
+ *   lowdiff_allgather_sparse  Sync(G~_{i,t})       Alg.1 line 5
+ *   lowdiff_batch_merge       batched C^B_t        §4.2 Step 2
+ *   lowdiff_stage_d2h         offload to CPU       §4.2 Step 1
+ *   lowdiff_replay            Recovery             Alg.1 lines 16-24, Eq.1
+ *
+ * Conventions (all calls):
+ *  - Pointers are DEVICE pointers unless the argument says "host". The caller owns every buffer
+ *    (device memory, pinned host memory, workspaces); the library allocates nothing on the
+ *    hot-path calls. Workspace sizes come from the *_workspace_size queries.
+ *  - Every call is asynchronous on the given stream (a cudaStream_t; NULL = legacy default
+ *    stream). Host-side argument validation is synchronous. Data-dependent counts (nnz, record
+ *    bytes) are written to caller DEVICE memory; only lowdiff_record_bytes synchronizes.
+ *  - Every call returns a lowdiff_status; nothing is thrown across the ABI. On failure,
+ *    lowdiff_last_error() returns a thread-local description.
+ *  - Device pointers to bulk arrays must be 16-byte aligned (EINVAL otherwise).
+ *  - Index width is u32; n must be < 2^31 (EINVAL otherwise; every BASELINE config fits:
+ *    GPT-2 XL has n = 1,557,611,200).
+ *  - Floating point: IEEE binary32, round-to-nearest-even per operation, no FMA contraction,
+ *    no flush-to-zero, fixed fold orders (rank-ascending, iteration-ascending), no float atomics:
+ *    results are deterministic and equal the CPU oracle's bit for bit.
+ */
+#ifndef LOWDIFF_H
+#define LOWDIFF_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st* lowdiff_stream_t; /* == cudaStream_t */
+
+typedef int32_t lowdiff_status;
+enum {
+  LOWDIFF_OK = 0,
+  LOWDIFF_EINVAL = 1,        /* bad argument (null/misaligned pointer, size, dtype, range)    */
+  LOWDIFF_EWORKSPACE = 2,    /* workspace smaller than the *_workspace_size query returned   */
+  LOWDIFF_ECAPACITY = 3,     /* an output (record, coalesced list) exceeds its capacity       */
+  LOWDIFF_ECHAIN = 4,        /* replay records not contiguous in t, or shard/n/nranks differ */
+  LOWDIFF_ECORRUPT = 5,      /* record bytes fail validation                                  */
+  LOWDIFF_EUNSUPPORTED = 6,  /* e.g. SUM record with momentum/Adam without opt-in             */
+  LOWDIFF_ECUDA = 7,         /* CUDA runtime error (message in lowdiff_last_error)            */
+  LOWDIFF_ENCCL = 8          /* NCCL error                                                    */
+};
+
+typedef enum { LOWDIFF_F32 = 0, LOWDIFF_BF16 = 1 } lowdiff_dtype;
+typedef enum { LOWDIFF_MERGE_SUM = 0, LOWDIFF_MERGE_STACK = 1 } lowdiff_merge_mode;
+typedef enum { LOWDIFF_OPT_SGD = 0, LOWDIFF_OPT_MOMENTUM = 1, LOWDIFF_OPT_ADAM = 2 } lowdiff_opt_kind;
+
+const char* lowdiff_status_string(lowdiff_status s);
+const char* lowdiff_last_error(void);      /* thread-local detail of the last failure       */
+const char* lowdiff_version(void);
+
+/* k = max(1, min(n, floor(rho * n))) evaluated in double — the number of pairs one rank emits
+ * at compression ratio rho (reading #2). */
+uint64_t lowdiff_k_for_density(uint64_t n, double rho);
+
+/* Bytes of one rank's packed pairs: pad16(4k) + pad16(sizeof(vdt) * k). */
+uint64_t lowdiff_pairs_bytes(uint64_t k, lowdiff_dtype vdt);
+
+/* Contiguous parameter-index shard owned by `rank` of `nranks`:
+ * [floor(rank n / nranks), floor((rank+1) n / nranks))   (reading #22). */
+lowdiff_status lowdiff_shard_bounds(uint64_t n, int32_t nranks, int32_t rank, uint64_t* lo, uint64_t* hi);
+
+/* ---------------------------------------------------------------------------------------------
+ * (1) Compress — Comp(G_{i,t}), Alg.1 line 4; "sparsification" at ratio rho.
+ *     Exact top-k with error feedback (north_star; readings #1-#8):
+ *       a = fp32(grad) + residual                         (one fp32 add; bf16 widening exact)
+ *       S = the k largest a by |a| (u32 key = bits(a) & 0x7FFFFFFF; equal keys: lower index first)
+ *       pairs = [ idx u32 x k ascending | zero pad to 16 B | val x k | zero pad to 16 B ]
+ *         vdt F32 : val = a[S];             residual <- a off S, +0 on S
+ *         vdt BF16: val = bf16_rne(a[S]);   residual <- a off S, a - fp32(val) on S (exact)
+ *   grad      [n] gdt (F32 or BF16), read only.      residual [n] fp32, updated in place.
+ *   pairs     lowdiff_pairs_bytes(k, vdt) bytes, written.   1 <= k <= n < 2^31.
+ *   ws        lowdiff_compress_workspace_size(n, k) bytes; contents need not be preserved.
+ * Errors: EINVAL (k, n, dtype, alignment), EWORKSPACE. The streaming pass is driven by a
+ * sampled threshold; if it under- or over-shoots, an exact full-array path runs on device
+ * (same result, more HBM traffic); nothing is reported to the host.
+ * ------------------------------------------------------------------------------------------- */
+lowdiff_status lowdiff_compress_workspace_size(uint64_t n, uint64_t k, uint64_t* bytes);
+lowdiff_status lowdiff_compress(const void* grad, lowdiff_dtype gdt, float* residual, uint64_t n,
+                                uint64_t k, void* pairs, lowdiff_dtype vdt, void* ws,
+                                uint64_t ws_bytes, lowdiff_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------------
+ * (2) Sparse all-gather + coalesce — Sync(G~_{i,t}), Alg.1 line 5; "Allgather".
+ *     Every rank passes its k pairs (same k and vdt on all ranks); ncclAllGather moves the fixed-
+ *     size packed buffers over NVLink; then the union of gathered indices within [lo, hi) is
+ *     coalesced: val = (rank-ascending fp32 fold) / P if `average`, else the fold. Zero sums are
+ *     kept (the index set is the union). Output: idx u32 ascending unique, val fp32, and the
+ *     count in *d_out_nnz (device u64). out_cap must be >= min(P*k, hi-lo) (else EINVAL).
+ *   comm == NULL means P = 1 (no collective; coalesce of the local list only).
+ * lowdiff_coalesce is the same coalesce over P packed buffers already resident on this device
+ * (laid out back to back, each lowdiff_pairs_bytes(k, vdt) long) — the post-gather half.
+ * ------------------------------------------------------------------------------------------- */
+typedef struct lowdiff_comm lowdiff_comm;
+int32_t        lowdiff_comm_unique_id_bytes(void);                 /* 128 */
+lowdiff_status lowdiff_comm_get_unique_id(uint8_t* id /* host, 128 bytes */);
+lowdiff_status lowdiff_comm_init(lowdiff_comm** comm, const uint8_t* id /* host */, int32_t nranks,
+                                 int32_t rank);  /* binds the calling thread's current device */
+lowdiff_status lowdiff_comm_destroy(lowdiff_comm* comm);
+
+lowdiff_status lowdiff_coalesce_workspace_size(int32_t nranks, uint64_t k, lowdiff_dtype vdt,
+                                               uint64_t lo, uint64_t hi, uint64_t* bytes);
+lowdiff_status lowdiff_coalesce(const void* gathered, int32_t nranks, uint64_t k, lowdiff_dtype vdt,
+                                uint64_t lo, uint64_t hi, int32_t average, uint32_t* out_idx,
+                                float* out_val, uint64_t out_cap, uint64_t* d_out_nnz, void* ws,
+                                uint64_t ws_bytes, lowdiff_stream_t stream);
+lowdiff_status lowdiff_allgather_sparse_workspace_size(int32_t nranks, uint64_t k, lowdiff_dtype vdt,
+                                                       uint64_t lo, uint64_t hi, uint64_t* bytes);
+lowdiff_status lowdiff_allgather_sparse(lowdiff_comm* comm, const void* pairs, uint64_t k,
+                                        lowdiff_dtype vdt, uint64_t lo, uint64_t hi, int32_t average,
+                                        uint32_t* out_idx, float* out_val, uint64_t out_cap,
+                                        uint64_t* d_out_nnz, void* ws, uint64_t ws_bytes,
+                                        lowdiff_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------------
+ * (3) Batch merge — Step 2 of batched gradient writing: B consecutive differentials of
+ *     one shard become one record C^B ("tensor addition or dictionary accumulation"):
+ *       SUM   (tensor addition):       U = union; val = iteration-ascending fp32 fold
+ *       STACK (dictionary accumulation): per u in U the (iteration, value) list, iteration order
+ *     The record layout (little-endian, every section 16-byte aligned, zero padding):
+ *       header (lowdiff_record_header, 80 B) | f32 lr[B] | u32 idx[nnz] |
+ *       SUM: f32 val[nnz]      STACK: u32 off[nnz+1] | u8 it[nent] | f32 val[nent]
+ *   diffs     HOST array of B views; idx/val/d_nnz are device pointers, `cap` bounds nnz (host).
+ *   d_record  record_cap bytes; d_record_bytes (device u64) receives the record's size.
+ *   1 <= B <= 255. The record never exceeds lowdiff_record_max_bytes(mode, B, sum of caps).
+ * ------------------------------------------------------------------------------------------- */
+typedef struct {
+  const uint32_t* idx;     /* device, ascending unique, lo <= idx < hi */
+  const float* val;        /* device */
+  const uint64_t* d_nnz;   /* device u64: number of entries */
+  uint64_t cap;            /* host: upper bound of *d_nnz */
+  float lr;                /* learning rate of this iteration (stored in the record's lr[]) */
+} lowdiff_diff_view;
+
+typedef struct {           /* == the first 80 bytes of every record */
+  uint8_t magic[8];        /* "LOWDIFF\x01" */
+  uint32_t version, mode, B, nranks;
+  uint64_t n, lo, hi, t_first, nnz, nent, total_bytes;
+} lowdiff_record_header;
+
+uint64_t       lowdiff_record_size(lowdiff_merge_mode mode, uint32_t B, uint64_t nnz, uint64_t nent);
+uint64_t       lowdiff_record_max_bytes(lowdiff_merge_mode mode, uint32_t B, uint64_t max_entries);
+lowdiff_status lowdiff_batch_merge_workspace_size(uint32_t B, uint64_t max_entries, uint64_t lo,
+                                                  uint64_t hi, uint64_t* bytes);
+lowdiff_status lowdiff_batch_merge(const lowdiff_diff_view* diffs /* host [B] */, uint32_t B,
+                                   lowdiff_merge_mode mode, uint64_t n, uint64_t lo, uint64_t hi,
+                                   uint64_t t_first, uint32_t nranks, void* d_record,
+                                   uint64_t record_cap, uint64_t* d_record_bytes, void* ws,
+                                   uint64_t ws_bytes, lowdiff_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------------
+ * (4) Stage — Step 1, `offload_to_cpu()` non-blocking.
+ *   lowdiff_record_bytes: synchronizes `stream`, reads *d_record_bytes; ECAPACITY if the merge
+ *     needed more than record_cap bytes (the record was not written).
+ *   lowdiff_stage_d2h: async copy of `bytes` record bytes into caller-owned pinned host memory
+ *     on copy_stream (a copy engine); byte-identical to the device record.
+ * ------------------------------------------------------------------------------------------- */
+lowdiff_status lowdiff_record_bytes(const uint64_t* d_record_bytes, uint64_t record_cap,
+                                    lowdiff_stream_t stream, uint64_t* bytes /* host */);
+lowdiff_status lowdiff_stage_d2h(const void* d_record, uint64_t bytes, void* h_pinned,
+                                 uint64_t h_cap, lowdiff_stream_t copy_stream);
+
+/* ---------------------------------------------------------------------------------------------
+ * (5) Replay — Recovery, Alg.1 lines 16-24: from a full checkpoint at iteration t,
+ *     apply the records of iterations t, t+1, ... in order. Each iteration is a DENSE optimizer
+ *     step with gradient 0 at absent indices (Comp^{-1}): SGD (x -= lr*(g + wd x)),
+ *     SGD-momentum (torch.optim.SGD conventions), Adam (Eq.1; bias-corrected, eps
+ *     after the sqrt). STACK records: one step per iteration (lr = lr[j]). SUM records: one step
+ *     with the summed gradient and lr[0] — exact trajectory only for SGD, so momentum/Adam
+ *     need allow_accumulated_sum (else EUNSUPPORTED); a SUM record's lr[] must be constant.
+ *     Scalars are computed on the host in double and rounded once to fp32.
+ *   recs[i].d_record: device record bytes; recs[i].h_head: HOST copy of (at least) its header
+ *     and lr[] (e.g. the pinned staging buffer); h_head_len >= 80 + 4B.
+ *   st: x (and m = momentum buffer or Adam m, v = Adam v) fp32 device arrays over [lo, hi),
+ *     x_bf16 optional device bf16 copy of x written after the last step; st->t, st->adam_step and
+ *     st->momentum_initialized are advanced on return (host fields).
+ * Errors: ECHAIN (t gap/overlap, n/lo/hi/nranks mismatch), ECORRUPT (header), EUNSUPPORTED.
+ * ------------------------------------------------------------------------------------------- */
+typedef struct {
+  int32_t kind;                       /* lowdiff_opt_kind */
+  double momentum, dampening, weight_decay, beta1, beta2, eps;
+  int32_t nesterov;
+  int32_t allow_accumulated_sum;
+} lowdiff_opt;
+
+typedef struct {
+  float* x; float* m; float* v; uint16_t* x_bf16;
+  uint64_t n, lo, hi;
+  uint64_t t;                         /* iteration whose G~ is applied next */
+  uint64_t adam_step;                 /* Adam step count stored in the full checkpoint */
+  int32_t momentum_initialized;
+} lowdiff_state;
+
+typedef struct {
+  const void* d_record;               /* device */
+  const void* h_head;                 /* host: header + lr[] (>= 80 + 4B bytes) */
+  uint64_t h_head_len;
+} lowdiff_record_view;
+
+lowdiff_status lowdiff_record_parse(const void* h_bytes, uint64_t len, lowdiff_record_header* out);
+lowdiff_status lowdiff_replay_workspace_size(const lowdiff_state* st, const lowdiff_record_view* recs,
+                                             uint32_t nrec, uint64_t* bytes);
+lowdiff_status lowdiff_replay(lowdiff_state* st, const lowdiff_opt* opt,
+                              const lowdiff_record_view* recs, uint32_t nrec, void* ws,
+                              uint64_t ws_bytes, lowdiff_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------------
+ * Instrumentation (bench/tests only; not on the data path).
+ *   lowdiff_launch_count: number of kernels this library has launched in the process.
+ *   lowdiff_profile_enable(1): from now on, bracket every launch of the named kernel classes
+ *     with CUDA events on the launching stream; lowdiff_profile_query sums the elapsed time
+ *     (synchronizing the events) of launches whose class name equals `name`, then forgets them.
+ *     Classes: "compress_stream", "compress_sample", "compress_select", "compress_emit",
+ *     "coalesce", "merge", "merge_pack", "replay_dense", "replay_sparse", "starts".
+ * ------------------------------------------------------------------------------------------- */
+uint64_t       lowdiff_launch_count(void);
+lowdiff_status lowdiff_profile_enable(int32_t on);
+lowdiff_status lowdiff_profile_query(const char* name, double* total_ms, uint64_t* launches);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LOWDIFF_H */

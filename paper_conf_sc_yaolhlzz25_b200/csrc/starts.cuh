@@ -1,0 +1,37 @@
+// Window-start index of sorted u32 lists (used by the merge engine and by replay).
+#pragma once
+#include "common.cuh"
+#include "internal.h"
+
+namespace lowdiff {
+
+__device__ __forceinline__ uint64_t list_len(const ListSet& ls, int l) {
+  return ls.list[l].d_len ? *ls.list[l].d_len : ls.list[l].len;
+}
+
+// starts[l*(num_w+1) + w] = first position e of list l with idx[e] >= lo + w*W (entries below
+// lo are skipped); starts[l*(num_w+1) + num_w] = first position with idx >= hi (or len).
+// One streaming pass over the entries: entry e writes the windows in (win(e-1), win(e)].
+template <int W>
+__global__ void __launch_bounds__(kThreads) starts_kernel(const __grid_constant__ ListSet ls, uint64_t lo,
+                                                          uint64_t hi, uint32_t num_w, uint32_t* starts) {
+  const int l = blockIdx.y;
+  const uint32_t* idx = ls.list[l].idx;
+  const uint64_t len = list_len(ls, l);
+  uint32_t* st = starts + (uint64_t)l * (num_w + 1);
+  auto win = [&](uint64_t e) -> int64_t {
+    if (e >= len) return (int64_t)num_w;
+    const uint64_t i = idx[e];
+    if (i < lo) return -1;
+    if (i >= hi) return (int64_t)num_w;
+    return (int64_t)((i - lo) / W);
+  };
+  for (uint64_t e = (uint64_t)blockIdx.x * kThreads + threadIdx.x; e <= len;
+       e += (uint64_t)gridDim.x * kThreads) {
+    const int64_t prev = (e == 0) ? -1 : win(e - 1);
+    const int64_t cur = win(e);
+    for (int64_t w = prev + 1; w <= cur; ++w) st[w] = (uint32_t)e;
+  }
+}
+
+}  // namespace lowdiff
