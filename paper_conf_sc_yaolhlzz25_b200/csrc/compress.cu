@@ -13,15 +13,20 @@
 // workloads). Nothing on this path is a dense contraction: no tensor cores.
 #include <stdio.h>
 
+#include <cooperative_groups.h>
+
 #include "common.cuh"
 #include "internal.h"
+
+namespace cg = cooperative_groups;
 
 namespace lowdiff {
 namespace {
 
 constexpr int kTile = 4096;            // elements per streaming tile: 256 thr x 4 vectors x 4
-constexpr int kTilesPerEmit = 32;      // streaming tiles per emission block (8 warps x 4)
+constexpr int kTilesPerEmit = kThreads; // streaming tiles per emission block (one per thread)
 constexpr int kSampleChunk = 1024;     // contiguous elements per sample chunk
+constexpr int kMaxSelectBlocks = 4 * 148;
 // digit p = (key >> shift(p)) & (bins(p) - 1): 12 + 10 + 9 bits of the 31-bit key
 __host__ __device__ constexpr int bins(int p) { return p == 0 ? 4096 : (p == 1 ? 1024 : 512); }
 __host__ __device__ constexpr int shift(int p) { return p == 0 ? 19 : (p == 1 ? 9 : 0); }
@@ -41,7 +46,7 @@ struct __align__(256) Ctl {
 };
 
 struct Layout {
-  uint64_t ctl, hs, h0, h1, h2, status, zero_end, tiles, cand_idx, cand_val, total;
+  uint64_t ctl, hs, h0, h1, h2, status, zero_end, tiles, cand_idx, cand_val, sloc, tloc, boff, total;
   uint32_t num_tiles, num_emit, cap;
 };
 
@@ -62,6 +67,9 @@ Layout layout(uint64_t n, uint64_t k) {
   L.tiles = o;    o += align256(8ull * L.num_tiles);
   L.cand_idx = o; o += align256(4ull * L.cap);
   L.cand_val = o; o += align256(4ull * L.cap);
+  L.sloc = o;     o += align256(8ull * (L.cap + 1));   // candidate flag scan
+  L.tloc = o;     o += align256(8ull * L.num_tiles);   // tile count scan
+  L.boff = o;     o += align256(8ull * 3 * kMaxSelectBlocks);
   L.total = o;
   return L;
 }
@@ -86,22 +94,29 @@ __device__ __forceinline__ float load_g1(const void* g, uint64_t i) {
 // ---- histogram "find": the bin holding the need-th largest key (1-based) --------------------
 // h: global histogram (nb bins, nb % 256 == 0). Walks bins from the top. Returns the bin
 // (or -1 if the total is below `need`) and, via *above, the count in strictly higher bins.
-__device__ int find_bin_desc(const uint32_t* h, int nb, uint64_t need, uint64_t* above_out,
-                             uint64_t* smem_scan) {
+template <int NB>
+__device__ int find_bin_desc(const uint32_t* h, uint64_t need, uint64_t* above_out, uint64_t* smem_scan) {
   __shared__ int s_bin;
   __shared__ uint64_t s_above;
-  const int per = nb / kThreads;
-  const int hi = nb - threadIdx.x * per;           // this thread's bins: [hi - per, hi)
+  constexpr int PER = NB / kThreads;               // 16, 4 or 2 bins per thread, loaded as vectors
+  const int lo = NB - (threadIdx.x + 1) * PER;     // this thread's bins: [lo, lo + PER)
+  uint32_t c[PER];
+#pragma unroll
+  for (int q = 0; q < PER; q += 2) {
+    const uint2 u = __ldcg(reinterpret_cast<const uint2*>(h + lo + q));
+    c[q] = u.x; c[q + 1] = u.y;
+  }
   uint64_t sum = 0;
-  for (int b = hi - 1; b >= hi - per; --b) sum += __ldcg(h + b);
+#pragma unroll
+  for (int q = 0; q < PER; ++q) sum += c[q];
   if (threadIdx.x == 0) { s_bin = -1; s_above = 0; }
   uint64_t total;
   uint64_t above = block_exclusive_scan(sum, smem_scan, &total);   // syncs inside
   if (above < need && above + sum >= need) {
-    for (int b = hi - 1; b >= hi - per; --b) {
-      uint32_t c = __ldcg(h + b);
-      if (above + c >= need) { s_bin = b; s_above = above; break; }
-      above += c;
+#pragma unroll
+    for (int q = PER - 1; q >= 0; --q) {
+      if (above + c[q] >= need) { s_bin = lo + q; s_above = above; break; }
+      above += c[q];
     }
   }
   __syncthreads();
@@ -120,20 +135,37 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(const void* g, const f
   __shared__ bool s_last;
   for (int b = threadIdx.x; b < bins(0); b += kThreads) sh[b] = 0;
   __syncthreads();
-  for (uint32_t c = blockIdx.x; c < num_chunks; c += gridDim.x) {
-    uint64_t start = exhaustive ? (uint64_t)c * kSampleChunk
-                                : (((uint64_t)c * (n - kSampleChunk)) / (num_chunks - 1)) & ~3ull;
-    uint64_t i = start + threadIdx.x * 4;
-    if (i + 3 < n) {
-      float4 gv = load_g4<BF16>(g, i);
-      float4 rv = *reinterpret_cast<const float4*>(r + i);
-      atomicAdd(&sh[mag_key(gv.x + rv.x) >> shift(0)], 1u);
-      atomicAdd(&sh[mag_key(gv.y + rv.y) >> shift(0)], 1u);
-      atomicAdd(&sh[mag_key(gv.z + rv.z) >> shift(0)], 1u);
-      atomicAdd(&sh[mag_key(gv.w + rv.w) >> shift(0)], 1u);
-    } else {
-      for (uint64_t j = i; j < i + 4 && j < n; ++j)
-        atomicAdd(&sh[mag_key(load_g1<BF16>(g, j) + r[j]) >> shift(0)], 1u);
+  // 4 chunks per round, loads issued before any use (memory-level parallelism)
+  auto chunk_start = [&](uint32_t c) -> uint64_t {
+    return exhaustive ? (uint64_t)c * kSampleChunk
+                      : (((uint64_t)c * (n - kSampleChunk)) / (num_chunks - 1)) & ~3ull;
+  };
+  for (uint32_t c0 = blockIdx.x; c0 < num_chunks; c0 += 4 * gridDim.x) {
+    float4 gv[4], rv[4];
+    bool vec[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint32_t c = c0 + u * gridDim.x;
+      const uint64_t i = c < num_chunks ? chunk_start(c) + threadIdx.x * 4 : n;
+      vec[u] = i + 3 < n;
+      if (vec[u]) {
+        gv[u] = load_g4<BF16>(g, i);
+        rv[u] = *reinterpret_cast<const float4*>(r + i);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint32_t c = c0 + u * gridDim.x;
+      if (vec[u]) {
+        atomicAdd(&sh[mag_key(gv[u].x + rv[u].x) >> shift(0)], 1u);
+        atomicAdd(&sh[mag_key(gv[u].y + rv[u].y) >> shift(0)], 1u);
+        atomicAdd(&sh[mag_key(gv[u].z + rv[u].z) >> shift(0)], 1u);
+        atomicAdd(&sh[mag_key(gv[u].w + rv[u].w) >> shift(0)], 1u);
+      } else if (c < num_chunks) {
+        const uint64_t i = chunk_start(c) + threadIdx.x * 4;
+        for (uint64_t j = i; j < i + 4 && j < n; ++j)
+          atomicAdd(&sh[mag_key(load_g1<BF16>(g, j) + r[j]) >> shift(0)], 1u);
+      }
     }
   }
   __syncthreads();
@@ -150,7 +182,7 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(const void* g, const f
   uint64_t S = exhaustive ? n : (uint64_t)num_chunks * kSampleChunk;
   uint64_t need = exhaustive ? k : (uint64_t)(1.15 * (double)k * (double)S / (double)n) + 8;
   uint64_t above;
-  int b = find_bin_desc(hs, bins(0), need, &above, s_scan);
+  int b = find_bin_desc<bins(0)>(hs, need, &above, s_scan);
   if (threadIdx.x == 0) {
     ctl->t_est = (b < 0) ? 0u : ((uint32_t)b << shift(0));
     ctl->k_rem = k;
@@ -254,55 +286,182 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
 }
 
 // ---- K1c: exact radix select over the candidates (or the full array) ------------------------
+// One cooperative launch runs the three digit passes (12 + 10 + 9 bits of the 31-bit key) with a
+// grid barrier after each histogram; every CTA then redoes the tiny 'find' on the L2-resident
+// histogram itself, so no second barrier or serial tail is needed per pass.
 template <int PASS>
-__global__ void __launch_bounds__(kThreads) select_kernel(const float* __restrict__ r, uint64_t n,
-                                                          uint64_t k, Ctl* ctl,
-                                                          const float* __restrict__ cand_val,
-                                                          uint32_t cap, uint32_t* hist) {
+__device__ __forceinline__ void select_pass(const float* __restrict__ src, uint64_t N, uint32_t* sh,
+                                            uint32_t* hist, uint32_t& prefix, uint64_t& need,
+                                            uint64_t* s_scan, cg::grid_group& grid) {
   constexpr int NB = bins(PASS);
   constexpr int SH = shift(PASS);
-  __shared__ uint32_t sh[NB];
-  __shared__ uint64_t s_scan[kThreads / 32];
-  __shared__ bool s_last;
   for (int b = threadIdx.x; b < NB; b += kThreads) sh[b] = 0;
-  uint32_t mode;
-  if (PASS == 0) {
-    const uint32_t cc = ctl->cand_count;
-    mode = (cc >= k && cc <= cap) ? 0u : 1u;
-  } else {
-    mode = ctl->mode;
-  }
-  const uint32_t prefix = (PASS == 0) ? 0u : ctl->prefix;
-  const float* src = mode ? r : cand_val;
-  const uint64_t N = mode ? n : (uint64_t)ctl->cand_count;
   __syncthreads();
-  for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < N;
-       i += (uint64_t)gridDim.x * kThreads) {
+  for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < N; i += (uint64_t)gridDim.x * kThreads) {
     const uint32_t key = mag_key(src[i]);
     if (PASS == 0 || (key >> shift(PASS > 0 ? PASS - 1 : 0)) == prefix) atomicAdd(&sh[(key >> SH) & (NB - 1)], 1u);
   }
   __syncthreads();
   for (int b = threadIdx.x; b < NB; b += kThreads)
     if (sh[b]) atomicAdd(hist + b, sh[b]);
-  __threadfence();
-  __syncthreads();
-  if (threadIdx.x == 0) s_last = (atomicAdd(&ctl->sel_ticket[PASS], 1u) == gridDim.x - 1);
-  __syncthreads();
-  if (!s_last) return;
-  __threadfence();
-  const uint64_t need = ctl->k_rem;
+  grid.sync();
   uint64_t above;
-  int d = find_bin_desc(hist, NB, need, &above, s_scan);
-  if (threadIdx.x == 0) {
-    ctl->count_gt += above;
-    ctl->k_rem = need - above;
-    if (PASS == 0) { ctl->mode = mode; ctl->prefix = (uint32_t)d; }
-    if (PASS == 1) ctl->prefix = (prefix << 10) | (uint32_t)d;
-    if (PASS == 2) { ctl->kstar = (prefix << 9) | (uint32_t)d; ctl->m = need - above; }
+  const int d = find_bin_desc<NB>(hist, need, &above, s_scan);
+  need -= above;
+  prefix = (PASS == 0) ? (uint32_t)d : ((prefix << (PASS == 1 ? 10 : 9)) | (uint32_t)d);
+  __syncthreads();
+}
+
+// Chunked block scan of packed (count > K*, count == K*) values over positions [a, e) of a block's
+// chunk: writes the block-local exclusive prefix to out[p]; returns the chunk total.
+template <typename ValueFn>
+__device__ __forceinline__ uint64_t chunk_scan(uint64_t a, uint64_t e, ValueFn value, uint64_t* out,
+                                               uint64_t* s_scan) {
+  uint64_t carry = 0;
+  for (uint64_t base = a; base < e; base += (uint64_t)kThreads * 4) {
+    uint64_t v[4], sum = 0;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const uint64_t p = base + threadIdx.x * 4 + j;
+      v[j] = p < e ? value(p) : 0;
+      sum += v[j];
+    }
+    uint64_t tot;
+    uint64_t run = carry + block_exclusive_scan(sum, s_scan, &tot);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const uint64_t p = base + threadIdx.x * 4 + j;
+      if (p < e) out[p] = run;
+      run += v[j];
+    }
+    carry += tot;
+  }
+  return carry;
+}
+
+// Exclusive prefix of the blocks' chunk totals (each block sums bsum[0, blockIdx.x)).
+__device__ __forceinline__ uint64_t block_offset(const uint64_t* bsum, uint64_t* s_scan) {
+  uint64_t part = 0;
+  for (uint32_t b = threadIdx.x; b < blockIdx.x; b += kThreads) part += __ldcg(bsum + b);
+  uint64_t tot;
+  block_exclusive_scan(part, s_scan, &tot);
+  return tot;
+}
+
+template <bool VBF16>
+__global__ void __launch_bounds__(kThreads) select_kernel(float* __restrict__ r, uint64_t n, uint64_t k,
+                                                          Ctl* ctl, const float* __restrict__ cand_val,
+                                                          const uint32_t* __restrict__ cand_idx,
+                                                          const uint2* __restrict__ tile_info,
+                                                          uint32_t num_tiles, uint32_t cap, uint32_t* h0,
+                                                          uint32_t* h1, uint32_t* h2, uint64_t* sloc,
+                                                          uint64_t* tloc, uint64_t* boff, uint8_t* pairs) {
+  cg::grid_group grid = cg::this_grid();
+  __shared__ uint32_t sh[bins(0)];
+  __shared__ uint64_t s_scan[kThreads / 32];
+  const uint32_t cc = ctl->cand_count;
+  const uint32_t mode = (cc >= k && cc <= cap) ? 0u : 1u;
+  const float* src = mode ? r : cand_val;
+  const uint64_t N = mode ? n : (uint64_t)cc;
+  uint32_t prefix = 0;
+  uint64_t need = k;
+  select_pass<0>(src, N, sh, h0, prefix, need, s_scan, grid);
+  select_pass<1>(src, N, sh, h1, prefix, need, s_scan, grid);
+  select_pass<2>(src, N, sh, h2, prefix, need, s_scan, grid);
+  const uint32_t K = prefix;
+  const uint64_t m = need;                         // K*-ties to keep (lowest indices first)
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    ctl->mode = mode;
+    ctl->kstar = K;
+    ctl->m = m;
+  }
+  if (mode != 0) return;                           // full-array fallback: emit_kernel does it
+  // ---- candidate mode: fused ordered emission ----
+  // (1) exclusive scan of packed (gt << 32 | eq) flags over the candidate buffer positions
+  const uint32_t G = gridDim.x, b = blockIdx.x;
+  const uint32_t cs = (uint32_t)((N + 1 + G - 1) / G);
+  const uint64_t a0 = (uint64_t)b * cs, a1 = (a0 + cs < N + 1) ? a0 + cs : N + 1;
+  auto flag = [&](uint64_t p) -> uint64_t {
+    if (p >= N) return 0;
+    const uint32_t key = mag_key(cand_val[p]);
+    return ((uint64_t)(key > K) << 32) | (uint64_t)(key == K);
+  };
+  const uint64_t stot = a0 < a1 ? chunk_scan(a0, a1, flag, sloc, s_scan) : 0;
+  if (threadIdx.x == 0) boff[b] = stot;
+  grid.sync();
+  const uint64_t soff = block_offset(boff, s_scan);
+  __syncthreads();
+  if (threadIdx.x == 0) boff[G + b] = soff;        // second half: per-block offsets
+  grid.sync();
+  auto S = [&](uint64_t p) -> uint64_t { return sloc[p] + __ldcg(boff + G + (uint32_t)p / cs); };
+  // (2) exclusive scan over tiles (index order) of the per-tile counts S(end) - S(begin)
+  const uint32_t ts = (num_tiles + G - 1) / G;
+  const uint64_t t0 = (uint64_t)b * ts, t1 = (t0 + ts < num_tiles) ? t0 + ts : num_tiles;
+  auto tcount = [&](uint64_t t) -> uint64_t {
+    const uint2 ti = tile_info[t];
+    return S((uint64_t)ti.x + ti.y) - S(ti.x);
+  };
+  const uint64_t ttot = t0 < t1 ? chunk_scan(t0, t1, tcount, tloc, s_scan) : 0;
+  grid.sync();                                     // everyone has read boff[b] (first half)
+  if (threadIdx.x == 0) boff[b] = ttot;
+  grid.sync();
+  const uint64_t toff = block_offset(boff, s_scan);
+  __syncthreads();
+  if (threadIdx.x == 0) boff[2 * G + b] = toff;
+  grid.sync();
+  // (3) every candidate finds its output position; selected ones are written (ascending index)
+  uint32_t* out_idx = reinterpret_cast<uint32_t*>(pairs);
+  uint8_t* out_val = pairs + pad16(4 * k);
+  if (b == 0 && threadIdx.x < 16) {                // zero the 16-byte padding of both sections
+    const uint64_t ip = 4 * k, ie = pad16(4 * k);
+    if (ip + threadIdx.x < ie) pairs[ip + threadIdx.x] = 0;
+    const uint64_t vp = pad16(4 * k) + (VBF16 ? 2 : 4) * k, ve = pad16(4 * k) + pad16((VBF16 ? 2 : 4) * k);
+    if (vp + threadIdx.x < ve) pairs[vp + threadIdx.x] = 0;
+  }
+  for (uint64_t i = (uint64_t)b * kThreads + threadIdx.x; i < N; i += (uint64_t)G * kThreads) {
+    const float a = cand_val[i];
+    const uint32_t key = mag_key(a);
+    if (key < K) continue;
+    const uint32_t idx = cand_idx[i];
+    const uint32_t t = idx / kTile;
+    const uint64_t tp = tloc[t] + __ldcg(boff + 2 * G + t / ts);
+    const uint64_t in_tile = S(i) - S(tile_info[t].x);
+    const uint64_t gtb = (tp >> 32) + (in_tile >> 32);
+    const uint64_t eqb = (tp & 0xFFFFFFFFull) + (in_tile & 0xFFFFFFFFull);
+    if (key > K || eqb < m) {
+      const uint64_t pos = gtb + (eqb < m ? eqb : m);
+      out_idx[pos] = idx;
+      if constexpr (VBF16) {
+        const __nv_bfloat16 h = __float2bfloat16_rn(a);
+        reinterpret_cast<__nv_bfloat16*>(out_val)[pos] = h;
+        r[idx] = a - __bfloat162float(h);          // exact (Sterbenz), reading #8
+      } else {
+        reinterpret_cast<float*>(out_val)[pos] = a;
+        r[idx] = 0.0f;
+      }
+    }
   }
 }
 
 // ---- K1d: ordered emission of the k pairs + residual fix-up on S ---------------------------
+// One CTA covers kTilesPerEmit = 256 streaming tiles. Candidate mode: one thread per tile walks its
+// (few) candidates; full mode (fallback): one warp per tile, 32 elements at a time. The per-tile
+// (count > K*, count == K*) pairs are scanned in the block and across blocks (decoupled look-back),
+// giving every selected element its output position gt_before + min(m, eq_before).
+template <bool VBF16>
+__device__ __forceinline__ void emit_one(uint64_t pos, uint32_t idx, float a, uint32_t* out_idx,
+                                         uint8_t* out_val, float* r) {
+  out_idx[pos] = idx;
+  if constexpr (VBF16) {
+    const __nv_bfloat16 h = __float2bfloat16_rn(a);
+    reinterpret_cast<__nv_bfloat16*>(out_val)[pos] = h;
+    r[idx] = a - __bfloat162float(h);              // exact (Sterbenz), reading #8
+  } else {
+    reinterpret_cast<float*>(out_val)[pos] = a;
+    r[idx] = 0.0f;
+  }
+}
+
 template <bool VBF16>
 __global__ void __launch_bounds__(kThreads) emit_kernel(float* __restrict__ r, uint64_t n, uint64_t k,
                                                         uint32_t num_tiles, uint32_t num_emit,
@@ -311,10 +470,12 @@ __global__ void __launch_bounds__(kThreads) emit_kernel(float* __restrict__ r, u
                                                         const float* __restrict__ cand_val,
                                                         uint64_t* status, uint8_t* pairs) {
   __shared__ uint32_t s_cnt[kTilesPerEmit][2];
-  __shared__ uint64_t s_pre[kTilesPerEmit];
+  __shared__ uint64_t s_scan[kThreads / 32];
+  __shared__ uint64_t s_bpre;
   __shared__ uint32_t s_ticket;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t mode = ctl->mode, K = ctl->kstar;
+  if (mode == 0) return;                           // candidate mode: emitted by select_kernel
   const uint64_t m = ctl->m;
   uint32_t* out_idx = reinterpret_cast<uint32_t*>(pairs);
   uint8_t* out_val = pairs + pad16(4 * k);
@@ -324,84 +485,89 @@ __global__ void __launch_bounds__(kThreads) emit_kernel(float* __restrict__ r, u
     __syncthreads();
     const uint32_t eb = s_ticket;
     if (eb >= num_emit) break;
-    if (eb == 0 && tid < 32) {               // zero the 16-byte padding of both sections
+    if (eb == 0 && tid < 16) {               // zero the 16-byte padding of both sections
       const uint64_t ip = 4 * k, ie = pad16(4 * k);
       if (ip + tid < ie) pairs[ip + tid] = 0;
       const uint64_t vp = pad16(4 * k) + (VBF16 ? 2 : 4) * k, ve = pad16(4 * k) + pad16((VBF16 ? 2 : 4) * k);
       if (vp + tid < ve) pairs[vp + tid] = 0;
     }
+    const uint32_t t_mine = eb * kTilesPerEmit + tid;
     // phase 1: per-tile counts of keys > K* and == K*
-#pragma unroll 1
-    for (int q = 0; q < 4; ++q) {
-      const uint32_t t = eb * kTilesPerEmit + warp * 4 + q;
-      uint32_t gt = 0, eq = 0;
-      if (t < num_tiles) {
-        uint64_t s, e;
-        if (mode == 0) { uint2 ti = tile_info[t]; s = ti.x; e = (uint64_t)ti.x + ti.y; }
-        else { s = (uint64_t)t * kTile; e = s + kTile < n ? s + kTile : n; }
-        const float* src = mode ? r : cand_val;
-        for (uint64_t i = s + lane; i < e; i += 32) {
-          const uint32_t key = mag_key(src[i]);
+    uint32_t gt = 0, eq = 0;
+    if (mode == 0) {
+      if (t_mine < num_tiles) {
+        const uint2 ti = tile_info[t_mine];
+        for (uint32_t i = ti.x; i < ti.x + ti.y; ++i) {
+          const uint32_t key = mag_key(cand_val[i]);
           gt += key > K; eq += key == K;
         }
       }
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) {
-        gt += __shfl_xor_sync(0xFFFFFFFFu, gt, o);
-        eq += __shfl_xor_sync(0xFFFFFFFFu, eq, o);
-      }
-      if (lane == 0) { s_cnt[warp * 4 + q][0] = gt; s_cnt[warp * 4 + q][1] = eq; }
-    }
-    __syncthreads();
-    if (warp == 0) {
-      const uint64_t v = ((uint64_t)s_cnt[lane][0] << 31) | s_cnt[lane][1];
-      uint64_t incl = v;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        uint64_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
-        if (lane >= o) incl += y;
-      }
-      const uint64_t tot = __shfl_sync(0xFFFFFFFFu, incl, 31);
-      const uint64_t bpre = lookback_exclusive(status, eb, tot);
-      s_pre[lane] = bpre + incl - v;
-    }
-    __syncthreads();
-    // phase 2: emit in index order
-#pragma unroll 1
-    for (int q = 0; q < 4; ++q) {
-      const uint32_t t = eb * kTilesPerEmit + warp * 4 + q;
-      if (t >= num_tiles) break;
-      uint64_t gtb = s_pre[warp * 4 + q] >> 31, eqb = s_pre[warp * 4 + q] & 0x7FFFFFFFull;
-      uint64_t s, e;
-      if (mode == 0) { uint2 ti = tile_info[t]; s = ti.x; e = (uint64_t)ti.x + ti.y; }
-      else { s = (uint64_t)t * kTile; e = s + kTile < n ? s + kTile : n; }
-      for (uint64_t i0 = s; i0 < e; i0 += 32) {
-        const uint64_t i = i0 + lane;
-        float a = 0.f;
-        uint32_t idx = 0;
-        bool valid = i < e;
-        if (valid) {
-          if (mode == 0) { a = cand_val[i]; idx = cand_idx[i]; }
-          else { a = r[i]; idx = (uint32_t)i; }
-        }
-        const uint32_t key = mag_key(a);
-        const bool isgt = valid && key > K, iseq = valid && key == K;
-        const uint32_t bg = __ballot_sync(0xFFFFFFFFu, isgt), be = __ballot_sync(0xFFFFFFFFu, iseq);
-        const uint64_t gb = gtb + __popc(bg & lt), eqbefore = eqb + __popc(be & lt);
-        if (isgt || (iseq && eqbefore < m)) {
-          const uint64_t pos = gb + (eqbefore < m ? eqbefore : m);
-          out_idx[pos] = idx;
-          if constexpr (VBF16) {
-            const __nv_bfloat16 h = __float2bfloat16_rn(a);
-            reinterpret_cast<__nv_bfloat16*>(out_val)[pos] = h;
-            r[idx] = a - __bfloat162float(h);          // exact (Sterbenz), reading #8
-          } else {
-            reinterpret_cast<float*>(out_val)[pos] = a;
-            r[idx] = 0.0f;
+    } else {
+      for (int q = 0; q < 32; ++q) {
+        const uint32_t t = eb * kTilesPerEmit + warp * 32 + q;
+        uint32_t g2 = 0, e2 = 0;
+        if (t < num_tiles) {
+          const uint64_t s = (uint64_t)t * kTile, e = s + kTile < n ? s + kTile : n;
+          for (uint64_t i = s + lane; i < e; i += 32) {
+            const uint32_t key = mag_key(r[i]);
+            g2 += key > K; e2 += key == K;
           }
         }
-        gtb += __popc(bg);
-        eqb += __popc(be);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+          g2 += __shfl_xor_sync(0xFFFFFFFFu, g2, o);
+          e2 += __shfl_xor_sync(0xFFFFFFFFu, e2, o);
+        }
+        if (lane == q) { gt = g2; eq = e2; }
+      }
+    }
+    uint64_t tot;
+    const uint64_t pre = block_exclusive_scan(((uint64_t)gt << 31) | eq, s_scan, &tot);
+    if (warp == 0) {
+      const uint64_t bpre = lookback_exclusive(status, eb, tot);
+      if (lane == 0) s_bpre = bpre;
+    }
+    __syncthreads();
+    const uint64_t mypre = s_bpre + pre;
+    // phase 2: emit in index order
+    if (mode == 0) {
+      if (t_mine < num_tiles) {
+        uint64_t gtb = mypre >> 31, eqb = mypre & 0x7FFFFFFFull;
+        const uint2 ti = tile_info[t_mine];
+        for (uint32_t i = ti.x; i < ti.x + ti.y; ++i) {
+          const float a = cand_val[i];
+          const uint32_t key = mag_key(a);
+          if (key > K) {
+            emit_one<VBF16>(gtb + (eqb < m ? eqb : m), cand_idx[i], a, out_idx, out_val, r);
+            ++gtb;
+          } else if (key == K) {
+            if (eqb < m) emit_one<VBF16>(gtb + eqb, cand_idx[i], a, out_idx, out_val, r);
+            ++eqb;
+          }
+        }
+      }
+    } else {
+      s_cnt[tid][0] = (uint32_t)(mypre >> 31);
+      s_cnt[tid][1] = (uint32_t)(mypre & 0x7FFFFFFFull);
+      __syncthreads();
+      for (int q = 0; q < 32; ++q) {
+        const uint32_t t = eb * kTilesPerEmit + warp * 32 + q;
+        if (t >= num_tiles) break;
+        uint64_t gtb = s_cnt[warp * 32 + q][0], eqb = s_cnt[warp * 32 + q][1];
+        const uint64_t s = (uint64_t)t * kTile, e = s + kTile < n ? s + kTile : n;
+        for (uint64_t i0 = s; i0 < e; i0 += 32) {
+          const uint64_t i = i0 + lane;
+          const bool valid = i < e;
+          const float a = valid ? r[i] : 0.f;
+          const uint32_t key = mag_key(a);
+          const bool isgt = valid && key > K, iseq = valid && key == K;
+          const uint32_t bg = __ballot_sync(0xFFFFFFFFu, isgt), be = __ballot_sync(0xFFFFFFFFu, iseq);
+          const uint64_t gb = gtb + __popc(bg & lt), eqbefore = eqb + __popc(be & lt);
+          if (isgt || (iseq && eqbefore < m))
+            emit_one<VBF16>(gb + (eqbefore < m ? eqbefore : m), (uint32_t)i, a, out_idx, out_val, r);
+          gtb += __popc(bg);
+          eqb += __popc(be);
+        }
       }
     }
     __syncthreads();
@@ -441,7 +607,7 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   const int exhaustive = (S >= n / 2) ? 1 : 0;
   const uint32_t chunks = exhaustive ? (uint32_t)((n + kSampleChunk - 1) / kSampleChunk)
                                      : (uint32_t)(S / kSampleChunk);
-  const int sample_grid = (int)(chunks < 1184u ? chunks : 1184u);
+  const int sample_grid = (int)(chunks < 2u * kNumSMs ? chunks : 2u * kNumSMs);
   uint32_t* hs = reinterpret_cast<uint32_t*>(w + L.hs);
   if (gdt == LOWDIFF_BF16)
     LD_LAUNCH("compress_sample", s, sample_kernel<true>, sample_grid, kThreads, 0, grad, residual, n,
@@ -463,13 +629,34 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
     LD_LAUNCH("compress_stream", s, stream_kernel<false>, grid, kThreads, 0, grad, residual, n,
               L.num_tiles, ctl, tiles, cidx, cval, L.cap);
 
-  const int sel_grid = 2 * kNumSMs;
-  LD_LAUNCH("compress_select", s, select_kernel<0>, sel_grid, kThreads, 0, residual, n, k, ctl, cval,
-            L.cap, reinterpret_cast<uint32_t*>(w + L.h0));
-  LD_LAUNCH("compress_select", s, select_kernel<1>, sel_grid, kThreads, 0, residual, n, k, ctl, cval,
-            L.cap, reinterpret_cast<uint32_t*>(w + L.h1));
-  LD_LAUNCH("compress_select", s, select_kernel<2>, sel_grid, kThreads, 0, residual, n, k, ctl, cval,
-            L.cap, reinterpret_cast<uint32_t*>(w + L.h2));
+  {
+    static int sel_grid = 0;
+    if (!sel_grid) {
+      int per_sm = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, select_kernel<false>, kThreads, 0);
+      int per_sm2 = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm2, select_kernel<true>, kThreads, 0);
+      if (per_sm2 < per_sm) per_sm = per_sm2;
+      sel_grid = (per_sm >= 2 ? 2 : 1) * kNumSMs;
+    }
+    float* rr = residual;
+    uint32_t *h0 = reinterpret_cast<uint32_t*>(w + L.h0), *h1 = reinterpret_cast<uint32_t*>(w + L.h1),
+             *h2 = reinterpret_cast<uint32_t*>(w + L.h2);
+    uint64_t* sloc = reinterpret_cast<uint64_t*>(w + L.sloc);
+    uint64_t* tloc = reinterpret_cast<uint64_t*>(w + L.tloc);
+    uint64_t* boff = reinterpret_cast<uint64_t*>(w + L.boff);
+    uint8_t* pp = static_cast<uint8_t*>(pairs);
+    const uint32_t* cidx_c = cidx;
+    const uint2* tiles_c = tiles;
+    uint32_t cap = L.cap, nt = L.num_tiles;
+    void* args[] = {(void*)&rr, (void*)&n, (void*)&k, (void*)&ctl, (void*)&cval, (void*)&cidx_c,
+                    (void*)&tiles_c, (void*)&nt, (void*)&cap, (void*)&h0, (void*)&h1, (void*)&h2,
+                    (void*)&sloc, (void*)&tloc, (void*)&boff, (void*)&pp};
+    ProfScope prof("compress_select", s);
+    const void* fn = vdt == LOWDIFF_BF16 ? (const void*)select_kernel<true> : (const void*)select_kernel<false>;
+    LD_CUDA(cudaLaunchCooperativeKernel(fn, sel_grid, kThreads, args, 0, s), "select launch");
+    note_launch();
+  }
 
   int egrid = (int)(L.num_emit < 4u * kNumSMs ? L.num_emit : 4u * kNumSMs);
   uint64_t* status = reinterpret_cast<uint64_t*>(w + L.status);

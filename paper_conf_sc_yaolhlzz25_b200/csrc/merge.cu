@@ -5,14 +5,26 @@
 //       accumulation") -> one record (SUM: iteration-ascending fold; STACK: per-index
 //       iteration lists)
 //
-// Sort-free design: the index range [lo, hi) is cut into windows of W = 4096
-// consecutive parameter indices. K2a writes, for every list, the position of each window's first
-// entry (one streaming pass over the entries). K2b is a persistent, ticket-ordered kernel: one
-// CTA takes one window, folds the lists' entries of that window into a dense W-slot
-// shared-memory accumulator IN LIST ORDER (so the fp32 fold order is the definition's, with no
-// float atomics), compacts the occupied slots in index order, and finds its global output offset
-// with a decoupled look-back. The merge writes sections into the workspace; K2c packs them into
-// the byte-exact record (header | lr[] | idx | val  or  off | it | val, 16-byte aligned).
+// Sort-free design. The index range [lo, hi) is cut into fine windows of
+// W = 4096 consecutive parameter indices.
+//   K2a  starts: for every list, the position of each fine window's first entry (one streaming
+//        pass over the entries).
+//   K2p  plan: consecutive fine windows are grouped G at a time (G from the host's density
+//        estimate, ~1K entries per group); a group whose entry count fits the shared-memory
+//        capacity becomes one "sparse" work item, a heavier group is split into its fine windows
+//        ("dense" items). Items are in index order.
+//   K2b  merge: persistent, ticket-ordered CTAs take one item each.
+//        sparse item: the lists' entries are loaded to shared memory and each entry's position
+//          in (index, list) order is computed by binary searches in the other lists' segments
+//          (the lists are sorted); runs of equal indices are folded in list order.
+//        dense item: the entries are folded into a W-slot shared-memory accumulator list by
+//          list, so the fp32 fold order is the definition's (rank / iteration ascending) with
+//          no float atomics, and occupied slots are compacted in index order.
+//        Items are independent: each writes its entries (STACK) at their final positions (the
+//        item's entry offset is the sum of its lists' start positions) and its unique heads to a
+//        staging array at that same offset.
+//   K2q  scan of the items' unique counts;  K2m  compaction of the staged heads.
+//   K2c  pack: sections -> the byte-exact record (header | lr[] | idx | val  or  off | it | val).
 #include "common.cuh"
 #include "internal.h"
 #include "starts.cuh"
@@ -20,18 +32,24 @@
 namespace lowdiff {
 namespace {
 
-constexpr int kW = 4096;                    // parameter indices per window
+constexpr int kW = 4096;                    // parameter indices per fine window
 constexpr int kSlotsPerThread = kW / kThreads;
+constexpr int kCap = 2048;                  // entries a sparse item may hold (shared memory)
+constexpr int kPosPerThread = kCap / kThreads;
+constexpr int kPlanThreads = 1024;
 
 struct __align__(256) MCtl {
   uint32_t ticket;
-  uint32_t pad;
-  uint64_t nnz;      // unique indices (written by the last window)
-  uint64_t nent;     // entries (STACK) (written by the last window)
+  uint32_t num_items;
+  uint64_t nnz;      // unique indices (written by the scan kernel)
+  uint64_t nent;     // entries (written by the scan kernel)
 };
 
+// Workspace. The merge kernel writes each item's unique heads into staging arrays at the item's
+// ENTRY offset (known from the starts table alone, so items need no ordering between them); a
+// scan over the items' unique counts and a compaction then place them densely.
 struct MLayout {
-  uint64_t ctl, status, zero_end, starts, widx, wval, woff, wit, went, total;
+  uint64_t ctl, zero_end, starts, items, ucnt, epre, upre, sidx, sval, widx, wval, wit, went, total;
   uint32_t num_w;
 };
 
@@ -41,14 +59,18 @@ MLayout mlayout(int L, uint64_t max_entries, uint64_t lo, uint64_t hi, bool reco
   const uint64_t cap_u = max_entries < hi - lo ? max_entries : hi - lo;
   uint64_t o = 0;
   M.ctl = o;    o += align256(sizeof(MCtl));
-  M.status = o; o += align256(8ull * M.num_w);
   M.zero_end = o;
   M.starts = o; o += align256(4ull * L * (M.num_w + 1));
-  M.widx = M.wval = M.woff = M.wit = M.went = 0;
+  M.items = o;  o += align256(8ull * M.num_w);
+  M.ucnt = o;   o += align256(4ull * M.num_w);   // unique count per item
+  M.epre = o;   o += align256(4ull * M.num_w);   // entry offset per item
+  M.upre = o;   o += align256(4ull * M.num_w);   // unique offset per item (scan)
+  M.sidx = o;   o += align256(4 * max_entries);  // staged heads: idx
+  M.sval = o;   o += align256(4 * max_entries);  // staged heads: value (SUM/coalesce) or off (STACK)
+  M.widx = M.wval = M.wit = M.went = 0;
   if (record) {
     M.widx = o; o += align256(4 * cap_u);
     M.wval = o; o += align256(4 * cap_u);         // SUM values, or STACK off[] (u32)
-    M.woff = M.wval;
     M.wit = o;  o += align256(max_entries);
     M.went = o; o += align256(4 * max_entries);
   }
@@ -64,127 +86,388 @@ __device__ __forceinline__ float list_val(const ListSet& ls, int l, uint64_t e) 
     return static_cast<const float*>(ls.list[l].val)[e];
 }
 
-// ---- K2b: window merge --------------------------------------------------------------------------
+// ---- K2p: work-item plan (one CTA) -----------------------------------------------------------------
+// items[i] = (first fine window, number of fine windows).
+__global__ void __launch_bounds__(kPlanThreads) plan_kernel(int L, const uint32_t* __restrict__ starts,
+                                                            uint32_t num_w, uint32_t G, MCtl* ctl,
+                                                            uint2* __restrict__ items) {
+  __shared__ uint32_t s_warp[kPlanThreads / 32];
+  __shared__ uint32_t s_carry;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t num_g = (num_w + G - 1) / G;
+  if (tid == 0) s_carry = 0;
+  __syncthreads();
+  for (uint32_t g0 = 0; g0 < num_g; g0 += kPlanThreads) {
+    const uint32_t g = g0 + tid;
+    uint32_t fs = 0, fe = 0, cnt = 0;
+    if (g < num_g) {
+      fs = g * G;
+      fe = fs + G < num_w ? fs + G : num_w;
+      uint64_t e = 0;
+      int l = 0;
+      for (; l + 4 <= L; l += 4) {                   // 8 independent loads in flight
+        uint32_t a[4], b[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const uint32_t* st = starts + (uint64_t)(l + q) * (num_w + 1);
+          a[q] = st[fe]; b[q] = st[fs];
+        }
+#pragma unroll
+        for (int q = 0; q < 4; ++q) e += a[q] - b[q];
+      }
+      for (; l < L; ++l) {
+        const uint32_t* st = starts + (uint64_t)l * (num_w + 1);
+        e += st[fe] - st[fs];
+      }
+      cnt = (e <= (uint64_t)kCap || fe - fs == 1) ? 1u : fe - fs;
+    }
+    uint32_t incl = cnt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+      if (lane >= o) incl += y;
+    }
+    if (lane == 31) s_warp[warp] = incl;
+    __syncthreads();
+    uint32_t off = s_carry, tot = 0;
+    for (int w = 0; w < kPlanThreads / 32; ++w) {
+      if (w < warp) off += s_warp[w];
+      tot += s_warp[w];
+    }
+    off += incl - cnt;
+    if (cnt == 1) items[off] = make_uint2(fs, fe - fs);
+    else
+      for (uint32_t s = 0; s < cnt; ++s) items[off + s] = make_uint2(fs + s, 1u);
+    __syncthreads();
+    if (tid == 0) s_carry += tot;
+    __syncthreads();
+  }
+  if (tid == 0) ctl->num_items = s_carry;
+}
+
+// ---- K2b: item merge ------------------------------------------------------------------------------
+struct DenseSmem {
+  float acc[kW];                 // SUM: running fold; STACK: slot entry cursor (u32)
+  uint32_t cnt[kW];              // entries per slot
+};
+struct SparseSmem {
+  uint64_t sk[kCap];             // (idx - w0) << 40 | list << 32 | load position; sorted in place
+  float val[kCap];               // values at their load position
+};
+union ItemSmem {
+  DenseSmem d;
+  SparseSmem s;
+};
+
 template <int KIND, bool BF16>
-__global__ void __launch_bounds__(kThreads) window_kernel(const __grid_constant__ ListSet ls, uint64_t lo,
-                                                          uint64_t hi, uint32_t num_w,
-                                                          const uint32_t* __restrict__ starts,
-                                                          MCtl* ctl, uint64_t* status, int average,
-                                                          uint32_t* __restrict__ out_idx,
-                                                          float* __restrict__ out_val,
-                                                          uint64_t* d_out_nnz,
-                                                          uint8_t* __restrict__ out_it,
-                                                          float* __restrict__ out_ent) {
-  __shared__ float s_acc[kW];                 // SUM: running fold; STACK: slot entry cursor (u32)
-  __shared__ uint32_t s_cnt[kW];              // entries per slot (lists present)
-  __shared__ uint32_t s_beg[kMaxLists], s_end[kMaxLists];
+__global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__ ListSet ls, uint64_t lo,
+                                                         uint32_t num_w, const uint32_t* __restrict__ starts,
+                                                         const uint2* __restrict__ items, MCtl* ctl,
+                                                         uint32_t* __restrict__ ucnt, uint32_t* __restrict__ epre,
+                                                         uint32_t* __restrict__ stg_idx,
+                                                         uint32_t* __restrict__ stg_val,
+                                                         uint8_t* __restrict__ out_it,
+                                                         float* __restrict__ out_ent) {
+  __shared__ ItemSmem sm;
+  __shared__ uint32_t s_beg[kMaxLists], s_len[kMaxLists], s_off[kMaxLists + 1];
   __shared__ uint64_t s_scan[kThreads / 32];
-  __shared__ uint64_t s_base;
-  __shared__ uint32_t s_ticket;
+  __shared__ uint32_t s_ticket, s_e0;
   const int tid = threadIdx.x;
   const int L = ls.L;
-  const float fP = (float)L;
-  for (int j = tid; j < kW; j += kThreads) s_cnt[j] = 0;
+  const uint32_t num_items = ctl->num_items;
+  for (int j = tid; j < kW; j += kThreads) sm.d.cnt[j] = 0;
+  bool dense_clean = true;                         // cnt[] is all zero
   while (true) {
     if (tid == 0) s_ticket = atomicAdd(&ctl->ticket, 1u);
     __syncthreads();
-    const uint32_t w = s_ticket;
-    if (w >= num_w) break;
-    const uint64_t w0 = lo + (uint64_t)w * kW;
-    int nonempty = 0;
-    for (int l = tid; l < L; l += kThreads) {
-      const uint32_t b = starts[(uint64_t)l * (num_w + 1) + w];
-      const uint32_t e = starts[(uint64_t)l * (num_w + 1) + w + 1];
-      s_beg[l] = b; s_end[l] = e;
-      nonempty |= (e > b);
+    const uint32_t item = s_ticket;
+    if (item >= num_items) break;
+    const uint2 it = items[item];
+    const uint64_t w0 = lo + (uint64_t)it.x * kW;
+    // per-list segments of this item; their prefix (list order); the item's entry offset
+    uint32_t len = 0, beg = 0;
+    if (tid < L) {
+      const uint32_t* st = starts + (uint64_t)tid * (num_w + 1);
+      beg = st[it.x];
+      len = st[it.x + it.y] - beg;
+      s_beg[tid] = beg;
+      s_len[tid] = len;
     }
-    nonempty = __syncthreads_or(nonempty);
-    uint64_t my_u = 0, my_e = 0, local = 0;
-    if (nonempty) {
+    uint64_t tot_e;
+    const uint64_t packed = block_exclusive_scan(((uint64_t)beg << 32) | len, s_scan, &tot_e);
+    if (tid < L) s_off[tid] = (uint32_t)packed;
+    if (tid == 0) {
+      s_off[L] = (uint32_t)tot_e;
+      s_e0 = (uint32_t)(tot_e >> 32);              // sum over lists of the item's first position
+    }
+    __syncthreads();
+    const uint32_t E = (uint32_t)tot_e;
+    const uint32_t e0 = s_e0;
+    uint64_t tot;
+    if (E <= (uint32_t)kCap) {
+      // ---- sparse item: load, then a shared-memory bitonic sort on the unique composite
+      //      (index, list) key — equal indices end up in list (rank / iteration) order ----
+      uint32_t Np = 32;
+      while (Np < E) Np <<= 1;
+      for (uint32_t x = tid; x < Np; x += kThreads) {
+        if (x < E) {
+          int a = 0, b = L - 1;                    // list l with s_off[l] <= x < s_off[l+1]
+          while (a < b) {
+            const int mid = (a + b + 1) >> 1;
+            if (s_off[mid] <= x) a = mid; else b = mid - 1;
+          }
+          const uint64_t e = s_beg[a] + (x - s_off[a]);
+          const uint32_t key = ls.list[a].idx[e] - (uint32_t)w0;
+          sm.s.sk[x] = ((uint64_t)key << 40) | ((uint64_t)a << 32) | x;
+          sm.s.val[x] = list_val<BF16>(ls, a, e);
+        } else {
+          sm.s.sk[x] = ~0ull;                      // padding sorts last
+        }
+      }
+      __syncthreads();
+      for (uint32_t kk = 2; kk <= Np; kk <<= 1) {
+        for (uint32_t j = kk >> 1; j > 0; j >>= 1) {
+          for (uint32_t i = tid; i < Np / 2; i += kThreads) {
+            const uint32_t lo_ = 2 * j * (i / j) + (i % j), hi_ = lo_ + j;
+            const uint64_t A = sm.s.sk[lo_], Bv = sm.s.sk[hi_];
+            if ((A > Bv) == ((lo_ & kk) == 0)) { sm.s.sk[lo_] = Bv; sm.s.sk[hi_] = A; }
+          }
+          __syncthreads();
+        }
+      }
+      uint32_t my_u = 0;
+#pragma unroll
+      for (int j = 0; j < kPosPerThread; ++j) {
+        const uint32_t r = tid * kPosPerThread + j;
+        if (r < E && (r == 0 || (sm.s.sk[r - 1] >> 40) != (sm.s.sk[r] >> 40))) ++my_u;
+      }
+      uint32_t u = e0 + (uint32_t)block_exclusive_scan(my_u, s_scan, &tot);
+#pragma unroll
+      for (int j = 0; j < kPosPerThread; ++j) {
+        const uint32_t r = tid * kPosPerThread + j;
+        if (r >= E) break;
+        const uint64_t skr = sm.s.sk[r];
+        const uint32_t key = (uint32_t)(skr >> 40);
+        const bool head = r == 0 || (sm.s.sk[r - 1] >> 40) != key;
+        if (KIND == kMergeStack) {
+          if (head) {
+            stg_idx[u] = (uint32_t)(w0 + key);
+            stg_val[u] = e0 + r;                   // off[] = the head's entry position
+            ++u;
+          }
+          out_it[e0 + r] = (uint8_t)(skr >> 32);
+          out_ent[e0 + r] = sm.s.val[(uint32_t)skr];
+        } else if (head) {
+          float sum = sm.s.val[(uint32_t)skr];     // fold the run in list order
+          for (uint32_t r2 = r + 1; r2 < E && (sm.s.sk[r2] >> 40) == key; ++r2)
+            sum = sum + sm.s.val[(uint32_t)sm.s.sk[r2]];
+          stg_idx[u] = (uint32_t)(w0 + key);
+          stg_val[u] = __float_as_uint(sum);
+          ++u;
+        }
+      }
+      dense_clean = false;                         // the sparse arrays alias cnt[]
+    } else {
+      // ---- dense item: exactly one fine window, any number of entries ----
+      if (!dense_clean) {
+        for (int j = tid; j < kW; j += kThreads) sm.d.cnt[j] = 0;
+        __syncthreads();
+      }
       if (KIND == kMergeStack) {
-        for (int l = 0; l < L; ++l)                     // integer counts: order-free
-          for (uint32_t e = s_beg[l] + tid; e < s_end[l]; e += kThreads)
-            atomicAdd(&s_cnt[ls.list[l].idx[e] - w0], 1u);
+        for (int l = 0; l < L; ++l)                // integer counts: order-free
+          for (uint32_t e = s_beg[l] + tid; e < s_beg[l] + s_len[l]; e += kThreads)
+            atomicAdd(&sm.d.cnt[ls.list[l].idx[e] - w0], 1u);
       } else {
-        for (int l = 0; l < L; ++l) {                   // fp32 fold in list (rank/iteration) order
-          if (s_end[l] == s_beg[l]) continue;           // block-uniform
-          for (uint32_t e = s_beg[l] + tid; e < s_end[l]; e += kThreads) {
+        for (int l = 0; l < L; ++l) {              // fp32 fold in list (rank/iteration) order
+          if (s_len[l] == 0) continue;             // block-uniform
+          for (uint32_t e = s_beg[l] + tid; e < s_beg[l] + s_len[l]; e += kThreads) {
             const uint32_t slot = ls.list[l].idx[e] - (uint32_t)w0;
             const float v = list_val<BF16>(ls, l, e);
-            const uint32_t c = s_cnt[slot];
-            s_acc[slot] = c ? s_acc[slot] + v : v;
-            s_cnt[slot] = c + 1;
+            const uint32_t c = sm.d.cnt[slot];
+            sm.d.acc[slot] = c ? sm.d.acc[slot] + v : v;
+            sm.d.cnt[slot] = c + 1;
           }
           __syncthreads();
         }
       }
       __syncthreads();
+      uint64_t my_u = 0, my_e = 0;
 #pragma unroll
       for (int j = 0; j < kSlotsPerThread; ++j) {
-        const uint32_t c = s_cnt[tid * kSlotsPerThread + j];
+        const uint32_t c = sm.d.cnt[tid * kSlotsPerThread + j];
         my_u += c ? 1 : 0;
         my_e += c;
       }
-      uint64_t tot;
-      local = block_exclusive_scan((my_u << 31) | my_e, s_scan, &tot);
-      if (tid < 32) {
-        const uint64_t pre = lookback_exclusive(status, w, tot);
-        if (tid == 0) s_base = pre;
-      }
-    } else {
-      if (tid < 32) {
-        const uint64_t pre = lookback_exclusive(status, w, 0);
-        if (tid == 0) s_base = pre;
-      }
-    }
-    __syncthreads();
-    const uint64_t base = s_base;
-    if (nonempty) {
-      uint64_t u = (base >> 31) + (local >> 31);
-      uint64_t e = (base & 0x7FFFFFFFull) + (local & 0x7FFFFFFFull);
+      const uint64_t local = block_exclusive_scan((my_u << 32) | my_e, s_scan, &tot);
+      uint32_t u = e0 + (uint32_t)(local >> 32);
+      uint32_t e = e0 + (uint32_t)local;
+      tot >>= 32;
 #pragma unroll 4
       for (int j = 0; j < kSlotsPerThread; ++j) {
         const int slot = tid * kSlotsPerThread + j;
-        const uint32_t c = s_cnt[slot];
+        const uint32_t c = sm.d.cnt[slot];
         if (!c) continue;
-        out_idx[u] = (uint32_t)(w0 + slot);
+        stg_idx[u] = (uint32_t)(w0 + slot);
         if (KIND == kMergeStack) {
-          reinterpret_cast<uint32_t*>(out_val)[u] = (uint32_t)e;      // off[u]
-          reinterpret_cast<uint32_t*>(s_acc)[slot] = (uint32_t)e;     // entry cursor
+          stg_val[u] = e;                                             // off[]
+          reinterpret_cast<uint32_t*>(sm.d.acc)[slot] = e;            // entry cursor
         } else {
-          const float s = s_acc[slot];
-          out_val[u] = average ? __fdiv_rn(s, fP) : s;
+          stg_val[u] = __float_as_uint(sm.d.acc[slot]);
         }
         ++u;
         e += c;
       }
       if (KIND == kMergeStack) {
         __syncthreads();
-        for (int l = 0; l < L; ++l) {                   // entries in iteration order per slot
-          if (s_end[l] == s_beg[l]) continue;
-          for (uint32_t x = s_beg[l] + tid; x < s_end[l]; x += kThreads) {
+        for (int l = 0; l < L; ++l) {              // entries in iteration order per slot
+          if (s_len[l] == 0) continue;
+          for (uint32_t x = s_beg[l] + tid; x < s_beg[l] + s_len[l]; x += kThreads) {
             const uint32_t slot = ls.list[l].idx[x] - (uint32_t)w0;
-            const uint32_t pos = reinterpret_cast<uint32_t*>(s_acc)[slot];
+            const uint32_t pos = reinterpret_cast<uint32_t*>(sm.d.acc)[slot];
             out_it[pos] = (uint8_t)l;
             out_ent[pos] = list_val<BF16>(ls, l, x);
-            reinterpret_cast<uint32_t*>(s_acc)[slot] = pos + 1;
+            reinterpret_cast<uint32_t*>(sm.d.acc)[slot] = pos + 1;
           }
           __syncthreads();
         }
       }
-      if (tid == kThreads - 1 && w == num_w - 1) {
-        ctl->nnz = u;
-        ctl->nent = e;
-        if (d_out_nnz) *d_out_nnz = u;
-      }
 #pragma unroll
-      for (int j = 0; j < kSlotsPerThread; ++j) s_cnt[tid * kSlotsPerThread + j] = 0;
-    } else if (tid == 0 && w == num_w - 1) {
-      ctl->nnz = base >> 31;
-      ctl->nent = base & 0x7FFFFFFFull;
-      if (d_out_nnz) *d_out_nnz = base >> 31;
+      for (int j = 0; j < kSlotsPerThread; ++j) sm.d.cnt[tid * kSlotsPerThread + j] = 0;
+      dense_clean = true;
+    }
+    if (tid == 0) {
+      ucnt[item] = (uint32_t)tot;
+      epre[item] = e0;
     }
     __syncthreads();
+  }
+}
+
+// ---- K2q: exclusive scan of the items' unique counts; totals (one CTA) ------------------------
+__global__ void __launch_bounds__(kPlanThreads) ucount_scan_kernel(const __grid_constant__ ListSet ls,
+                                                                   uint32_t num_w,
+                                                                   const uint32_t* __restrict__ starts,
+                                                                   MCtl* ctl, const uint32_t* __restrict__ ucnt,
+                                                                   uint32_t* __restrict__ upre,
+                                                                   uint64_t* d_out_nnz) {
+  __shared__ uint32_t s_warp[kPlanThreads / 32];
+  __shared__ uint32_t s_carry;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t num_items = ctl->num_items;
+  if (tid == 0) s_carry = 0;
+  __syncthreads();
+  for (uint32_t i0 = 0; i0 < num_items; i0 += kPlanThreads) {
+    const uint32_t i = i0 + tid;
+    const uint32_t c = i < num_items ? ucnt[i] : 0u;
+    uint32_t incl = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+      if (lane >= o) incl += y;
+    }
+    if (lane == 31) s_warp[warp] = incl;
+    __syncthreads();
+    uint32_t off = s_carry, tot = 0;
+    for (int w = 0; w < kPlanThreads / 32; ++w) {
+      if (w < warp) off += s_warp[w];
+      tot += s_warp[w];
+    }
+    if (i < num_items) upre[i] = off + incl - c;
+    __syncthreads();
+    if (tid == 0) s_carry += tot;
+    __syncthreads();
+  }
+  if (tid == 0) {
+    uint64_t nent = 0;
+    for (int l = 0; l < ls.L; ++l) {
+      const uint32_t* st = starts + (uint64_t)l * (num_w + 1);
+      nent += st[num_w] - st[0];
+    }
+    ctl->nnz = s_carry;
+    ctl->nent = nent;
+    if (d_out_nnz) *d_out_nnz = s_carry;
+  }
+}
+
+// ---- K2m: compaction of the staged heads (one warp per item) ----------------------------------
+__global__ void __launch_bounds__(kThreads) compact_kernel(const MCtl* ctl, const uint32_t* __restrict__ ucnt,
+                                                           const uint32_t* __restrict__ epre,
+                                                           const uint32_t* __restrict__ upre,
+                                                           const uint32_t* __restrict__ stg_idx,
+                                                           const uint32_t* __restrict__ stg_val,
+                                                           float inv_div, int divide, uint32_t* __restrict__ out_idx,
+                                                           uint32_t* __restrict__ out_val) {
+  const uint32_t num_items = ctl->num_items;
+  const int lane = threadIdx.x & 31;
+  (void)inv_div;
+  for (uint32_t i = (blockIdx.x * kThreads + threadIdx.x) >> 5; i < num_items; i += (gridDim.x * kThreads) >> 5) {
+    const uint32_t c = ucnt[i], src = epre[i], dst = upre[i];
+    for (uint32_t x0 = 0; x0 < c; x0 += 128) {       // 4 loads in flight per lane
+      uint32_t iv[4], vv[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint32_t x = x0 + q * 32 + lane;
+        if (x < c) { iv[q] = stg_idx[src + x]; vv[q] = stg_val[src + x]; }
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint32_t x = x0 + q * 32 + lane;
+        if (x >= c) break;
+        uint32_t v = vv[q];
+        if (divide) v = __float_as_uint(__fdiv_rn(__uint_as_float(v), inv_div));   // "/ P" (coalesce)
+        out_idx[dst + x] = iv[q];
+        out_val[dst + x] = v;
+      }
+    }
+  }
+}
+
+// ---- K2s: coalesce of a single list (P = 1): the union is the list itself, /1 is exact --------
+// Warp-parallel lower bound (32 probes per round) of `v` in a sorted list of `len`.
+__device__ uint64_t warp_lower_bound(const uint32_t* idx, uint64_t len, uint64_t v) {
+  const int lane = threadIdx.x & 31;
+  uint64_t lo = 0, hi = len;                       // answer in [lo, hi]
+  while (hi - lo > 32) {
+    const uint64_t step = (hi - lo + 31) / 32;
+    const uint64_t p = lo + (uint64_t)lane * step;
+    const bool less = p < hi && (uint64_t)idx[p] < v;
+    const uint32_t m = __ballot_sync(0xFFFFFFFFu, less);
+    const int c = __popc(m);                       // probes below v (a prefix of the lanes)
+    const uint64_t nlo = c ? lo + (uint64_t)(c - 1) * step + 1 : lo;
+    const uint64_t nhi = lo + (uint64_t)c * step;
+    lo = nlo;
+    hi = nhi < hi ? nhi : hi;
+  }
+  const uint64_t p = lo + lane;
+  const bool less = p < hi && (uint64_t)idx[p] < v;
+  return lo + __popc(__ballot_sync(0xFFFFFFFFu, less));
+}
+
+template <bool BF16>
+__global__ void __launch_bounds__(kThreads) single_list_kernel(const uint32_t* __restrict__ idx,
+                                                               const void* __restrict__ val, uint64_t len,
+                                                               uint64_t lo, uint64_t hi,
+                                                               uint32_t* __restrict__ out_idx,
+                                                               float* __restrict__ out_val,
+                                                               uint64_t* d_out_nnz) {
+  __shared__ uint64_t s_first, s_last;
+  if (threadIdx.x < 32) {
+    const uint64_t f = (len == 0 || idx[0] >= lo) ? 0 : warp_lower_bound(idx, len, lo);
+    const uint64_t l = (len == 0 || idx[len - 1] < hi) ? len : warp_lower_bound(idx, len, hi);
+    if (threadIdx.x == 0) {
+      s_first = f;
+      s_last = l;
+      if (blockIdx.x == 0) *d_out_nnz = l - f;
+    }
+  }
+  __syncthreads();
+  const uint64_t first = s_first, cnt = s_last - s_first;
+  for (uint64_t e = (uint64_t)blockIdx.x * kThreads + threadIdx.x; e < cnt; e += (uint64_t)gridDim.x * kThreads) {
+    out_idx[e] = idx[first + e];
+    float v;
+    if constexpr (BF16) v = __uint_as_float(((uint32_t) static_cast<const uint16_t*>(val)[first + e]) << 16);
+    else v = static_cast<const float*>(val)[first + e];
+    out_val[e] = __fdiv_rn(v, 1.0f);               // the definition's "/ P" with P = 1 (exact)
   }
 }
 
@@ -294,41 +577,67 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
                          uint64_t* d_record_bytes, void* ws, cudaStream_t s) {
   (void)out_cap;
   const bool record = kind != kCoalesce;
+  if (kind == kCoalesce && ls.L == 1) {
+    uint64_t g = (ls.list[0].len + kThreads - 1) / kThreads;
+    if (g > 4ull * kNumSMs) g = 4ull * kNumSMs;
+    if (g < 1) g = 1;
+    if (ls.bf16)
+      LD_LAUNCH("coalesce", s, single_list_kernel<true>, (int)g, kThreads, 0, ls.list[0].idx, ls.list[0].val,
+                ls.list[0].len, lo, hi, out_idx, out_val, d_out_nnz);
+    else
+      LD_LAUNCH("coalesce", s, single_list_kernel<false>, (int)g, kThreads, 0, ls.list[0].idx, ls.list[0].val,
+                ls.list[0].len, lo, hi, out_idx, out_val, d_out_nnz);
+    return cuda_status(cudaGetLastError(), "coalesce launch");
+  }
   const MLayout M = mlayout(ls.L, max_entries, lo, hi, record);
   uint8_t* w = static_cast<uint8_t*>(ws);
   MCtl* ctl = reinterpret_cast<MCtl*>(w + M.ctl);
-  uint64_t* status = reinterpret_cast<uint64_t*>(w + M.status);
   uint32_t* starts = reinterpret_cast<uint32_t*>(w + M.starts);
+  uint2* items = reinterpret_cast<uint2*>(w + M.items);
   LD_CUDA(cudaMemsetAsync(w, 0, M.zero_end, s), "memset merge workspace");
 
   uint64_t per_list = max_entries / (ls.L ? ls.L : 1) + 1;
   uint64_t gx = (per_list + kThreads - 1) / kThreads;
-  if (gx > 512) gx = 512;
+  if (gx > 8ull * kNumSMs) gx = 8ull * kNumSMs;
   if (gx < 1) gx = 1;
   LD_LAUNCH("starts", s, starts_kernel<kW>, dim3((unsigned)gx, (unsigned)ls.L), kThreads, 0, ls, lo, hi,
             M.num_w, starts);
 
-  const int grid = (int)(M.num_w < 4u * kNumSMs ? M.num_w : 4u * kNumSMs);
-  uint32_t* oidx = record ? reinterpret_cast<uint32_t*>(w + M.widx) : out_idx;
-  float* oval = record ? reinterpret_cast<float*>(w + M.wval) : out_val;
+  // group size: about kCap/2 entries per group at the average density (power of two)
+  const double per_w = (double)max_entries / (double)M.num_w;
+  uint32_t G = 1;
+  while (G < 4096 && (double)(2 * G) * per_w <= kCap / 2) G <<= 1;     // key < 2^24
+  LD_LAUNCH("merge_plan", s, plan_kernel, 1, kPlanThreads, 0, ls.L, starts, M.num_w, G, ctl, items);
+
+  const int grid = (int)(M.num_w < 3u * kNumSMs ? M.num_w : 3u * kNumSMs);
+  uint32_t* ucnt = reinterpret_cast<uint32_t*>(w + M.ucnt);
+  uint32_t* epre = reinterpret_cast<uint32_t*>(w + M.epre);
+  uint32_t* upre = reinterpret_cast<uint32_t*>(w + M.upre);
+  uint32_t* sidx = reinterpret_cast<uint32_t*>(w + M.sidx);
+  uint32_t* sval = reinterpret_cast<uint32_t*>(w + M.sval);
   uint8_t* oit = record ? w + M.wit : nullptr;
   float* oent = record ? reinterpret_cast<float*>(w + M.went) : nullptr;
   const char* cls = record ? "merge" : "coalesce";
-  if (kind == kCoalesce) {
-    if (ls.bf16)
-      LD_LAUNCH(cls, s, (window_kernel<kCoalesce, true>), grid, kThreads, 0, ls, lo, hi, M.num_w,
-                starts, ctl, status, average, oidx, oval, d_out_nnz, oit, oent);
-    else
-      LD_LAUNCH(cls, s, (window_kernel<kCoalesce, false>), grid, kThreads, 0, ls, lo, hi, M.num_w,
-                starts, ctl, status, average, oidx, oval, d_out_nnz, oit, oent);
-    return cuda_status(cudaGetLastError(), "coalesce launch");
-  }
-  if (kind == kMergeSum)
-    LD_LAUNCH(cls, s, (window_kernel<kMergeSum, false>), grid, kThreads, 0, ls, lo, hi, M.num_w,
-              starts, ctl, status, 0, oidx, oval, nullptr, oit, oent);
+  if (kind == kCoalesce && ls.bf16)
+    LD_LAUNCH(cls, s, (merge_kernel<kCoalesce, true>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
+              ucnt, epre, sidx, sval, oit, oent);
+  else if (kind == kCoalesce)
+    LD_LAUNCH(cls, s, (merge_kernel<kCoalesce, false>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
+              ucnt, epre, sidx, sval, oit, oent);
+  else if (kind == kMergeSum)
+    LD_LAUNCH(cls, s, (merge_kernel<kMergeSum, false>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
+              ucnt, epre, sidx, sval, oit, oent);
   else
-    LD_LAUNCH(cls, s, (window_kernel<kMergeStack, false>), grid, kThreads, 0, ls, lo, hi, M.num_w,
-              starts, ctl, status, 0, oidx, oval, nullptr, oit, oent);
+    LD_LAUNCH(cls, s, (merge_kernel<kMergeStack, false>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
+              ucnt, epre, sidx, sval, oit, oent);
+  LD_LAUNCH(cls, s, ucount_scan_kernel, 1, kPlanThreads, 0, ls, M.num_w, starts, ctl, ucnt, upre,
+            kind == kCoalesce ? d_out_nnz : nullptr);
+  uint32_t* didx = record ? reinterpret_cast<uint32_t*>(w + M.widx) : out_idx;
+  uint32_t* dval = record ? reinterpret_cast<uint32_t*>(w + M.wval) : reinterpret_cast<uint32_t*>(out_val);
+  const int cgrid = (int)((M.num_w + 7) / 8 < 4u * kNumSMs ? (M.num_w + 7) / 8 : 4u * kNumSMs);
+  LD_LAUNCH(cls, s, compact_kernel, cgrid, kThreads, 0, ctl, ucnt, epre, upre, sidx, sval, (float)ls.L,
+            (kind == kCoalesce && average) ? 1 : 0, didx, dval);
+  if (kind == kCoalesce) return cuda_status(cudaGetLastError(), "coalesce launch");
 
   PackArgs pa;
   pa.mode = kind == kMergeSum ? LOWDIFF_MERGE_SUM : LOWDIFF_MERGE_STACK;

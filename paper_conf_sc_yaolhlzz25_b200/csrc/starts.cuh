@@ -26,11 +26,29 @@ __global__ void __launch_bounds__(kThreads) starts_kernel(const __grid_constant_
     if (i >= hi) return (int64_t)num_w;
     return (int64_t)((i - lo) / W);
   };
-  for (uint64_t e = (uint64_t)blockIdx.x * kThreads + threadIdx.x; e <= len;
-       e += (uint64_t)gridDim.x * kThreads) {
-    const int64_t prev = (e == 0) ? -1 : win(e - 1);
-    const int64_t cur = win(e);
-    for (int64_t w = prev + 1; w <= cur; ++w) st[w] = (uint32_t)e;
+  // Short runs of windows are written by the entry's own lane; long gaps (sparse lists leave
+  // thousands of empty windows between entries) are written by the whole warp, coalesced.
+  const int lane = threadIdx.x & 31;
+  const uint64_t stride = (uint64_t)gridDim.x * kThreads;
+  for (uint64_t e0 = (uint64_t)blockIdx.x * kThreads + (threadIdx.x & ~31u); e0 <= len; e0 += stride) {
+    const uint64_t e = e0 + lane;
+    int64_t prev = 0, cur = -1;
+    if (e <= len) {
+      prev = (e == 0) ? -1 : win(e - 1);
+      cur = win(e);
+    }
+    const bool longr = cur - prev > 8;
+    if (!longr)
+      for (int64_t w = prev + 1; w <= cur; ++w) st[w] = (uint32_t)e;
+    uint32_t lm = __ballot_sync(0xFFFFFFFFu, longr);
+    while (lm) {
+      const int src = __ffs(lm) - 1;
+      lm &= lm - 1;
+      const int64_t from = __shfl_sync(0xFFFFFFFFu, prev, src) + 1;
+      const int64_t to = __shfl_sync(0xFFFFFFFFu, cur, src);
+      const uint32_t ee = (uint32_t)__shfl_sync(0xFFFFFFFFu, (unsigned long long)e, src);
+      for (int64_t w = from + lane; w <= to; w += 32) st[w] = ee;
+    }
   }
 }
 
