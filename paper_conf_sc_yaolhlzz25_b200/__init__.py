@@ -261,25 +261,34 @@ def coalesce(gathered: torch.Tensor, nranks: int, k: int, vdt="f32", lo: int = 0
     return out_idx, out_val, d_nnz
 
 
+def broadcast_bytes(data: bytes | None, nbytes: int, group=None) -> bytes:
+    """Rank 0's `data` (nbytes long) on every rank of the torch.distributed group (host plumbing for
+    the NCCL unique id; works on the nccl and gloo backends)."""
+    import torch.distributed as dist
+    t = torch.zeros(nbytes, dtype=torch.uint8)
+    if data is not None:
+        t.copy_(torch.frombuffer(bytearray(data), dtype=torch.uint8))
+    if dist.is_initialized() and dist.get_world_size(group) > 1:
+        dev = "cuda" if dist.get_backend(group) == "nccl" else "cpu"
+        td = t.to(dev)
+        dist.broadcast(td, src=0, group=group)
+        t = td.cpu()
+    return bytes(t.tolist())
+
+
 class Comm:
     """NCCL communicator of liblowdiff, bootstrapped through torch.distributed (the unique id is
     broadcast from rank 0 over the default process group)."""
 
     def __init__(self, nranks: int, rank: int, group=None):
-        import torch.distributed as dist
         self.nranks, self.rank = nranks, rank
         nid = int(lib().lowdiff_comm_unique_id_bytes())
-        uid = torch.zeros(nid, dtype=torch.uint8)
+        data = None
         if rank == 0:
             buf = (C.c_uint8 * nid)()
             _check(lib().lowdiff_comm_get_unique_id(buf), "comm_get_unique_id")
-            uid.copy_(torch.frombuffer(bytearray(buf), dtype=torch.uint8))
-        if nranks > 1:
-            dev = "cuda" if dist.get_backend(group) == "nccl" else "cpu"
-            t = uid.to(dev)
-            dist.broadcast(t, src=0, group=group)
-            uid = t.cpu()
-        raw = (C.c_uint8 * nid)(*uid.tolist())
+            data = bytes(buf)
+        raw = (C.c_uint8 * nid)(*broadcast_bytes(data, nid, group))
         self._h = C.c_void_p()
         _check(lib().lowdiff_comm_init(C.byref(self._h), raw, nranks, rank), "comm_init")
 
