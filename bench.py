@@ -45,8 +45,7 @@ def parse_args():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--profile-steps", type=int, default=-1,
-                    help="steps whose kernels are bracketed by CUDA events (-1: all timed steps)")
+    ap.add_argument("--no-graph", action="store_true", help="time eager launches (no CUDA graph)")
     return ap.parse_args()
 
 
@@ -204,8 +203,8 @@ def run_ours(args, cfg):
     copy_stream = torch.cuda.Stream()
     t_iter = [0]
 
-    def step(inputs=None, h2d=None):
-        """One pass of the path over one batch; returns staged record bytes."""
+    def build_phase(h2d=None):
+        """B iterations of compress -> sparse all-gather + coalesce of this rank's shard -> ring."""
         for j in range(B):
             if h2d is not None:               # e2e: this iteration's gradient from pinned host memory
                 h2d[0][j % len(h2d[0])].copy_(h2d[1][j % len(h2d[1])], non_blocking=True)
@@ -214,6 +213,9 @@ def run_ours(args, cfg):
                 g = grads[j]
             ld.compress(g, r, k, vdt=cfg.vdt, pairs=pairs)
             ld.allgather_sparse(comm, pairs, k, cfg.vdt, lo, hi, True, *ring[j])
+
+    def checkpoint_phase():
+        """Batch merge -> record -> D2H stage (copy stream) -> replay of the record; returns bytes."""
         diffs = [(ring[j][0], ring[j][1], ring[j][2], cap, lr) for j in range(B)]
         ld.batch_merge(diffs, cfg.merge, n, lo, hi, t_iter[0], P, record=record, d_record_bytes=d_bytes)
         nb = ld.record_bytes(d_bytes, rec_cap)          # the checkpoint thread's only sync
@@ -226,6 +228,14 @@ def run_ours(args, cfg):
         main.wait_stream(copy_stream)
         t_iter[0] += B
         return nb
+
+    def step(graph=None, h2d=None):
+        """One pass of the path over one batch."""
+        if graph is not None:
+            graph.replay()
+        else:
+            build_phase(h2d)
+        return checkpoint_phase()
 
     def timed(nsteps, **kw):
         if world > 1:
@@ -246,18 +256,41 @@ def run_ours(args, cfg):
             dist.barrier()
         return ms, nb
 
+    def capture(h2d=None):
+        """The build phase as one CUDA graph (launch-latency removal); None if capture fails."""
+        if args.no_graph:
+            return None, 0
+        try:
+            torch.cuda.synchronize()
+            g = torch.cuda.CUDAGraph()
+            l0 = ld.launch_count()
+            with torch.cuda.graph(g):
+                build_phase(h2d)
+            return g, ld.launch_count() - l0
+        except Exception as e:                           # pragma: no cover
+            print(f"graph capture failed ({e}); timing eager launches", file=sys.stderr)
+            torch.cuda.synchronize()
+            return None, 0
+
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
+    graph, graph_launches = capture()
+    if graph is not None:
+        step(graph=graph)                               # warm the graph once
+        torch.cuda.synchronize()
 
+    # ---- timed region (value): the whole path, build phase as a graph ----
     clocks = ClockSampler(local)
     clocks.start()
     launches0 = ld.launch_count()
-    ld.profile_enable(True)
-    ms, rec_bytes = timed(args.steps)
-    ld.profile_enable(False)
-    launches = ld.launch_count() - launches0
+    ms, rec_bytes = timed(args.steps, graph=graph)
+    launches = ld.launch_count() - launches0 + (graph_launches * args.steps if graph is not None else 0)
     clk = clocks.stop()
+    # ---- profiled pass (same work, eager launches, CUDA events around every kernel) ----
+    ld.profile_enable(True)
+    pms, _ = timed(args.steps)
+    ld.profile_enable(False)
     prof = {c: ld.profile_query(c) for c in ("compress_stream", "compress_sample", "compress_select",
                                              "compress_emit", "coalesce", "starts", "merge", "merge_pack",
                                              "replay_dense", "replay_sparse")}
@@ -297,9 +330,11 @@ def run_ours(args, cfg):
         dpool = [torch.empty_like(grads[0]) for _ in range(npool)]
         del grads
         torch.cuda.empty_cache()
-        step(h2d=(dpool, hpool))
+        eg, _ = capture(h2d=(dpool, hpool))
+        kw = {"graph": eg} if eg is not None else {"h2d": (dpool, hpool)}
+        step(**kw)
         e_steps = max(1, min(args.steps, 3))
-        ems, enb = timed(e_steps, h2d=(dpool, hpool))
+        ems, enb = timed(e_steps, **kw)
         e_ms = ems / e_steps
         e2e = {"value": P * B * n * gsz / (e_ms * 1e-3) / 1e9, "unit": "GB/s",
                "h2d_bytes_per_step": B * n * gsz, "d2h_bytes_per_step": int(enb) + 80 + 4 * B + 8,
@@ -325,6 +360,9 @@ def run_ours(args, cfg):
                            "differentials_per_s": P * B / (ms_step * 1e-3),
                            "replayed_iterations_per_s": B / (ms_step * 1e-3),
                            "record_bytes": int(rec_bytes)},
+                "timing": {"build_phase": "one CUDA graph per step" if graph is not None else "eager launches",
+                           "profiled_ms_per_step": pms / args.steps,
+                           "profiled": "separate pass, eager launches, CUDA events around every kernel"},
                 "roofline": roofline, "kernels": kernels, "cpu_baseline": cpu, "e2e": e2e,
                 "gpu_launches": int(launches), "clocks": clk}
         print(json.dumps(line), flush=True)

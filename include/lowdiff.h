@@ -227,6 +227,14 @@ lowdiff_status lowdiff_replay(lowdiff_state* st, const lowdiff_opt* opt,
  *     "coalesce", "merge", "merge_pack", "replay_dense", "replay_sparse", "starts".
  * ------------------------------------------------------------------------------------------- */
 uint64_t       lowdiff_launch_count(void);
+/* After a lowdiff_compress on `stream` with workspace `ws` (syncs the stream): out6 = {sampled
+ * threshold key, candidates found, path (0 = candidate buffer, 1 = full-array fallback), k-th key,
+ * ties kept, candidate capacity}. Diagnostics for tests and the bench. */
+lowdiff_status lowdiff_compress_stats(const void* ws, uint64_t n, uint64_t k, lowdiff_stream_t stream,
+                                      uint64_t* out6);
+/* Test hook: while enabled, every later lowdiff_compress uses `key` as its candidate threshold
+ * instead of the sampled estimate (to force the exact full-array fallback in tests). */
+lowdiff_status lowdiff_debug_force_threshold(int32_t enable, uint32_t key);
 lowdiff_status lowdiff_profile_enable(int32_t on);
 lowdiff_status lowdiff_profile_query(const char* name, double* total_ms, uint64_t* launches);
 

@@ -75,7 +75,8 @@ EXPORTS = [
     "lowdiff_record_size", "lowdiff_record_max_bytes", "lowdiff_batch_merge_workspace_size",
     "lowdiff_batch_merge", "lowdiff_record_bytes", "lowdiff_stage_d2h", "lowdiff_record_parse",
     "lowdiff_replay_workspace_size", "lowdiff_replay", "lowdiff_launch_count",
-    "lowdiff_profile_enable", "lowdiff_profile_query",
+    "lowdiff_profile_enable", "lowdiff_profile_query", "lowdiff_compress_stats",
+    "lowdiff_debug_force_threshold",
 ]
 
 _lib = None
@@ -121,6 +122,8 @@ def lib() -> C.CDLL:
         "lowdiff_launch_count": ([], u64),
         "lowdiff_profile_enable": ([i32], i32),
         "lowdiff_profile_query": ([C.c_char_p, vp, vp], i32),
+        "lowdiff_compress_stats": ([vp, u64, u64, vp, vp], i32),
+        "lowdiff_debug_force_threshold": ([i32, C.c_uint32], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -152,7 +155,10 @@ _ws_cache: dict = {}
 
 
 def workspace(nbytes: int, device, tag: str = "ws") -> torch.Tensor:
-    key = (str(torch.device(device)), tag)
+    d = torch.device(device)
+    if d.type == "cuda" and d.index is None:
+        d = torch.device("cuda", torch.cuda.current_device())
+    key = (str(d), tag)
     buf = _ws_cache.get(key)
     if buf is None or buf.numel() < nbytes:
         buf = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=device)
@@ -428,6 +434,20 @@ def replay(state: dict, opt: dict, records, ws=None, stream=None) -> dict:
 
 
 # ---- instrumentation --------------------------------------------------------------------------------
+def compress_stats(n: int, k: int, device="cuda", stream=None) -> dict:
+    """Diagnostics of the last compress that used the cached workspace (syncs the stream)."""
+    ws = workspace(compress_workspace_size(n, k), device, "compress")
+    out = (C.c_uint64 * 6)()
+    _check(lib().lowdiff_compress_stats(_cuda(ws, "ws"), n, k, _stream(stream), out), "compress_stats")
+    return dict(zip(("t_est", "candidates", "fallback", "kstar", "ties_kept", "capacity"), list(out)))
+
+
+def debug_force_threshold(key: int | None):
+    """Test hook: force the compress candidate threshold (None restores the sampled estimate)."""
+    _check(lib().lowdiff_debug_force_threshold(0 if key is None else 1, 0 if key is None else key),
+           "debug_force_threshold")
+
+
 def launch_count() -> int:
     return int(lib().lowdiff_launch_count())
 

@@ -445,6 +445,17 @@ lowdiff_status lowdiff_replay(lowdiff_state* st, const lowdiff_opt* opt, const l
 // ---- instrumentation ------------------------------------------------------------------------------
 uint64_t lowdiff_launch_count(void) { return g_launches.load(); }
 
+lowdiff_status lowdiff_debug_force_threshold(int32_t enable, uint32_t key) {
+  compress_force_threshold(enable, key);
+  return LOWDIFF_OK;
+}
+
+lowdiff_status lowdiff_compress_stats(const void* ws, uint64_t n, uint64_t k, lowdiff_stream_t stream,
+                                      uint64_t* out6) {
+  if (!ws || !out6) return fail(LOWDIFF_EINVAL, "compress_stats: null");
+  return compress_stats(ws, n, k, out6, (cudaStream_t)stream);
+}
+
 lowdiff_status lowdiff_profile_enable(int32_t on) {
   std::lock_guard<std::mutex> lk(g_prof_mu);
   g_prof_on = on != 0;

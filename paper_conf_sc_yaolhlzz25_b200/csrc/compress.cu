@@ -25,7 +25,6 @@ namespace {
 
 constexpr int kTile = 4096;            // elements per streaming tile: 256 thr x 4 vectors x 4
 constexpr int kTilesPerEmit = kThreads; // streaming tiles per emission block (one per thread)
-constexpr int kSampleChunk = 1024;     // contiguous elements per sample chunk
 constexpr int kMaxSelectBlocks = 4 * 148;
 // digit p = (key >> shift(p)) & (bins(p) - 1): 12 + 10 + 9 bits of the 31-bit key
 __host__ __device__ constexpr int bins(int p) { return p == 0 ? 4096 : (p == 1 ? 1024 : 512); }
@@ -54,7 +53,7 @@ Layout layout(uint64_t n, uint64_t k) {
   Layout L;
   L.num_tiles = (uint32_t)((n + kTile - 1) / kTile);
   L.num_emit = (L.num_tiles + kTilesPerEmit - 1) / kTilesPerEmit;
-  uint64_t cap = 4 * k + 65536;
+  uint64_t cap = 8 * k + 65536;
   L.cap = (uint32_t)(cap < n ? cap : n);
   uint64_t o = 0;
   L.ctl = o;      o += align256(sizeof(Ctl));
@@ -126,46 +125,37 @@ __device__ int find_bin_desc(const uint32_t* h, uint64_t need, uint64_t* above_o
 }
 
 // ---- K1a: stratified sample of keys -> threshold estimate ----------------------------------
+// Samples are 8-element (32-byte, sector-aligned) micro-chunks spread evenly over [0, n) with a
+// per-call phase, so small parameter segments are represented in proportion (coarse contiguous
+// chunks over-/under-represent segments smaller than their spacing, which biased the tail).
+// Exhaustive mode (small n) visits every micro-chunk.
 template <bool BF16>
 __global__ void __launch_bounds__(kThreads) sample_kernel(const void* g, const float* r, uint64_t n,
-                                                          uint64_t k, uint32_t num_chunks,
-                                                          int exhaustive, Ctl* ctl, uint32_t* hs) {
+                                                          uint64_t k, uint32_t num_micro, double stride,
+                                                          double phase, int exhaustive, Ctl* ctl,
+                                                          uint32_t* hs, uint32_t force_t) {
   __shared__ uint32_t sh[bins(0)];
   __shared__ uint64_t s_scan[kThreads / 32];
   __shared__ bool s_last;
   for (int b = threadIdx.x; b < bins(0); b += kThreads) sh[b] = 0;
   __syncthreads();
-  // 4 chunks per round, loads issued before any use (memory-level parallelism)
-  auto chunk_start = [&](uint32_t c) -> uint64_t {
-    return exhaustive ? (uint64_t)c * kSampleChunk
-                      : (((uint64_t)c * (n - kSampleChunk)) / (num_chunks - 1)) & ~3ull;
-  };
-  for (uint32_t c0 = blockIdx.x; c0 < num_chunks; c0 += 4 * gridDim.x) {
-    float4 gv[4], rv[4];
-    bool vec[4];
+  const uint64_t n8 = n / 8;
+  for (uint32_t m = blockIdx.x * kThreads + threadIdx.x; m < num_micro; m += gridDim.x * kThreads) {
+    uint64_t c8 = exhaustive ? m : (uint64_t)(((double)m + phase) * stride);
+    if (!exhaustive && c8 >= n8) c8 = n8 ? n8 - 1 : 0;
+    const uint64_t i = c8 * 8;
+    if (i + 8 <= n) {
+      float a[8];
+      const float4 r0 = *reinterpret_cast<const float4*>(r + i);
+      const float4 r1 = *reinterpret_cast<const float4*>(r + i + 4);
+      const float4 g0 = load_g4<BF16>(g, i);
+      const float4 g1 = load_g4<BF16>(g, i + 4);
+      a[0] = g0.x + r0.x; a[1] = g0.y + r0.y; a[2] = g0.z + r0.z; a[3] = g0.w + r0.w;
+      a[4] = g1.x + r1.x; a[5] = g1.y + r1.y; a[6] = g1.z + r1.z; a[7] = g1.w + r1.w;
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const uint32_t c = c0 + u * gridDim.x;
-      const uint64_t i = c < num_chunks ? chunk_start(c) + threadIdx.x * 4 : n;
-      vec[u] = i + 3 < n;
-      if (vec[u]) {
-        gv[u] = load_g4<BF16>(g, i);
-        rv[u] = *reinterpret_cast<const float4*>(r + i);
-      }
-    }
-#pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const uint32_t c = c0 + u * gridDim.x;
-      if (vec[u]) {
-        atomicAdd(&sh[mag_key(gv[u].x + rv[u].x) >> shift(0)], 1u);
-        atomicAdd(&sh[mag_key(gv[u].y + rv[u].y) >> shift(0)], 1u);
-        atomicAdd(&sh[mag_key(gv[u].z + rv[u].z) >> shift(0)], 1u);
-        atomicAdd(&sh[mag_key(gv[u].w + rv[u].w) >> shift(0)], 1u);
-      } else if (c < num_chunks) {
-        const uint64_t i = chunk_start(c) + threadIdx.x * 4;
-        for (uint64_t j = i; j < i + 4 && j < n; ++j)
-          atomicAdd(&sh[mag_key(load_g1<BF16>(g, j) + r[j]) >> shift(0)], 1u);
-      }
+      for (int e = 0; e < 8; ++e) atomicAdd(&sh[mag_key(a[e]) >> shift(0)], 1u);
+    } else {
+      for (uint64_t j = i; j < n; ++j) atomicAdd(&sh[mag_key(load_g1<BF16>(g, j) + r[j]) >> shift(0)], 1u);
     }
   }
   __syncthreads();
@@ -177,14 +167,36 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(const void* g, const f
   __syncthreads();
   if (!s_last) return;
   __threadfence();
-  // Need: exhaustive -> exactly k; sampled -> 1.15 x the expected sample count above the k-th
-  // key (+8), so the candidate count lands at >= ~1.15 k with a >5 sigma margin (S >= 2048 n/k).
-  uint64_t S = exhaustive ? n : (uint64_t)num_chunks * kSampleChunk;
-  uint64_t need = exhaustive ? k : (uint64_t)(1.15 * (double)k * (double)S / (double)n) + 8;
+  // Need: exhaustive -> exactly k (threshold = the bin's lower edge: exact, >= k candidates);
+  // sampled -> 1.3 x the expected sample count above the k-th key (+8): the candidates land at
+  // ~1.3 k, >8 sigma above k for S >= 2048 n / k. Within the 12.5 %-wide bin the threshold is
+  // placed by an exponential-density model fitted to this bin and the next one up (the tail
+  // density falls steeply, so a uniform model lands too high), then moved 10 % toward the lower
+  // edge as a safety margin.
+  uint64_t S = exhaustive ? n : (uint64_t)num_micro * 8;
+  uint64_t need = exhaustive ? k : (uint64_t)(1.3 * (double)k * (double)S / (double)n) + 8;
   uint64_t above;
   int b = find_bin_desc<bins(0)>(hs, need, &above, s_scan);
   if (threadIdx.x == 0) {
-    ctl->t_est = (b < 0) ? 0u : ((uint32_t)b << shift(0));
+    uint32_t t = (b < 0) ? 0u : ((uint32_t)b << shift(0));
+    if (b >= 0 && !exhaustive) {
+      const double c0 = (double)__ldcg(hs + b);
+      const double c1 = (b + 1 < bins(0)) ? (double)__ldcg(hs + b + 1) : 0.0;
+      const double f = (double)(need - above) / (c0 > 0 ? c0 : 1.0);   // share of the bin needed, (0, 1]
+      double x;                                                        // position from the bin's bottom
+      if (c1 >= c0 || c0 < 2) {
+        x = 1.0 - f;
+      } else {
+        const double lam = log(c0 / (c1 > 0.5 ? c1 : 0.5));
+        const double el = exp(-lam);
+        x = -log(f * (1.0 - el) + el) / lam;
+      }
+      x = 0.9 * (x < 0 ? 0 : (x > 1 ? 1 : x));
+      uint32_t off = (uint32_t)(x * (double)(1u << shift(0)));
+      if (off >= (1u << shift(0))) off = (1u << shift(0)) - 1;
+      t += off;
+    }
+    ctl->t_est = (force_t != 0xFFFFFFFFu) ? force_t : t;   // force_t: test hook
     ctl->k_rem = k;
   }
 }
@@ -575,6 +587,7 @@ __global__ void __launch_bounds__(kThreads) emit_kernel(float* __restrict__ r, u
 }
 
 int g_stream_blocks_f32 = 0, g_stream_blocks_bf16 = 0;
+uint32_t g_force_t = 0xFFFFFFFFu;       // test hook: override the sampled threshold
 
 int stream_blocks(bool bf16) {
   int& cache = bf16 ? g_stream_blocks_bf16 : g_stream_blocks_f32;
@@ -594,6 +607,18 @@ int stream_blocks(bool bf16) {
 
 uint64_t compress_ws_bytes(uint64_t n, uint64_t k) { return layout(n, k).total; }
 
+void compress_force_threshold(int enable, uint32_t key) { g_force_t = enable ? key : 0xFFFFFFFFu; }
+
+lowdiff_status compress_stats(const void* ws, uint64_t n, uint64_t k, uint64_t out[6], cudaStream_t s) {
+  (void)n; (void)k;
+  Ctl c;
+  LD_CUDA(cudaMemcpyAsync(&c, ws, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "stats copy");
+  LD_CUDA(cudaStreamSynchronize(s), "stats sync");
+  out[0] = c.t_est; out[1] = c.cand_count; out[2] = c.mode; out[3] = c.kstar; out[4] = c.m;
+  out[5] = layout(n, k).cap;
+  return LOWDIFF_OK;
+}
+
 lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t n, uint64_t k,
                             void* pairs, int vdt, void* ws, cudaStream_t s) {
   const Layout L = layout(n, k);
@@ -605,16 +630,20 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   uint64_t S = 65536;
   while ((double)S * (double)k < 2048.0 * (double)n && S < (1ull << 26)) S <<= 1;
   const int exhaustive = (S >= n / 2) ? 1 : 0;
-  const uint32_t chunks = exhaustive ? (uint32_t)((n + kSampleChunk - 1) / kSampleChunk)
-                                     : (uint32_t)(S / kSampleChunk);
-  const int sample_grid = (int)(chunks < 2u * kNumSMs ? chunks : 2u * kNumSMs);
+  const uint32_t micro = exhaustive ? (uint32_t)((n + 7) / 8) : (uint32_t)(S / 8);
+  const double stride = exhaustive ? 1.0 : (double)(n / 8) / (double)micro;
+  static uint64_t calls = 0;                       // per-call phase (golden-ratio sequence)
+  const double phase = exhaustive ? 0.0 : (double)((++calls * 0x9E3779B97F4A7C15ull) >> 11) * 0x1p-53;
+  uint64_t sg = (micro + kThreads - 1) / kThreads;
+  if (sg > 2ull * kNumSMs) sg = 2ull * kNumSMs;
+  const int sample_grid = (int)sg;
   uint32_t* hs = reinterpret_cast<uint32_t*>(w + L.hs);
   if (gdt == LOWDIFF_BF16)
     LD_LAUNCH("compress_sample", s, sample_kernel<true>, sample_grid, kThreads, 0, grad, residual, n,
-              k, chunks, exhaustive, ctl, hs);
+              k, micro, stride, phase, exhaustive, ctl, hs, g_force_t);
   else
     LD_LAUNCH("compress_sample", s, sample_kernel<false>, sample_grid, kThreads, 0, grad, residual,
-              n, k, chunks, exhaustive, ctl, hs);
+              n, k, micro, stride, phase, exhaustive, ctl, hs, g_force_t);
 
   uint2* tiles = reinterpret_cast<uint2*>(w + L.tiles);
   uint32_t* cidx = reinterpret_cast<uint32_t*>(w + L.cand_idx);

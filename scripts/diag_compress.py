@@ -1,0 +1,36 @@
+"""Diagnostics: sampled threshold quality over many EF iterations of a workload (GPU).
+
+    python scripts/diag_compress.py [--config 3] [--iters 300] [--cycle 16]
+Prints, every few iterations, the candidates found vs k, the capacity, and whether the exact
+full-array fallback ran.
+"""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch  # noqa: E402
+
+import paper_conf_sc_yaolhlzz25_b200 as ld  # noqa: E402
+from workloads import CONFIGS, gradient, segment_sigmas  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--config", type=int, default=3)
+ap.add_argument("--iters", type=int, default=300)
+ap.add_argument("--cycle", type=int, default=16)
+a = ap.parse_args()
+cfg = CONFIGS[a.config]
+dev = torch.device("cuda", 0)
+sig = segment_sigmas(cfg, dev)
+grads = [gradient(cfg, 0, t, dev, sigmas=sig) for t in range(a.cycle)]
+r = torch.zeros(cfg.n, device=dev)
+fallbacks = 0
+for it in range(a.iters):
+    ld.compress(grads[it % a.cycle], r, cfg.k, vdt=cfg.vdt)
+    st = ld.compress_stats(cfg.n, cfg.k)
+    fallbacks += st["fallback"]
+    if it < 20 or it % 16 == 0 or st["fallback"]:
+        print(f"it {it:4d} cand/k {st['candidates'] / cfg.k:7.3f} cap/k {st['capacity'] / cfg.k:6.2f} "
+              f"fallback {st['fallback']} t_est {st['t_est']:#x} kstar {st['kstar']:#x}", flush=True)
+print(f"fallbacks: {fallbacks} / {a.iters}")
