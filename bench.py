@@ -185,9 +185,14 @@ def run_ours(args, cfg):
     grads = [gradient(cfg, rank, t, dev, sigmas=sig) for t in range(B)]
     del sig
     r = torch.zeros(n, device=dev)
+    # Full checkpoint C^F shard (resident) and the recovered state M: every step's replay is one
+    # recovery, Load(C^F_t) + replay of the batch's record (Alg.1 l.16-24), read from the checkpoint
+    # and written to the state buffers (out of place: same HBM traffic as in place).
     ck = full_checkpoint(cfg, lo, hi, dev)
-    state = {"x": ck["x"], "m": ck["m"], "v": ck["v"], "x_bf16": None, "n": n, "lo": lo, "hi": hi,
-             "t": 0, "adam_step": ck["adam_step"], "momentum_initialized": ck["momentum_initialized"]}
+    state = {"x0": ck["x"], "m0": ck["m"], "v0": ck["v"],
+             "x": torch.empty_like(ck["x"]), "m": None if ck["m"] is None else torch.empty_like(ck["m"]),
+             "v": None if ck["v"] is None else torch.empty_like(ck["v"]), "x_bf16": None, "n": n, "lo": lo,
+             "hi": hi, "t": 0, "adam_step": ck["adam_step"], "momentum_initialized": ck["momentum_initialized"]}
     opt = {"kind": cfg.opt, **{kk: vv for kk, vv in cfg.hyper.items() if kk != "lr"}}
     lr = float(np.float32(cfg.hyper["lr"]))
     cap = min(P * k, hi - lo)
@@ -223,7 +228,9 @@ def run_ours(args, cfg):
         copy_stream.wait_stream(main)
         ld.stage_d2h(record, nb, staged, copy_stream)   # async persist staging (copy engine)
         main.synchronize()
-        state["t"] = t_iter[0]
+        state["t"] = t_iter[0]                          # the checkpoint is stamped at this batch's start
+        state["adam_step"] = ck["adam_step"]
+        state["momentum_initialized"] = ck["momentum_initialized"]
         ld.replay(state, opt, [(record, head)])
         main.wait_stream(copy_stream)
         t_iter[0] += B

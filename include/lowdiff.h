@@ -187,6 +187,9 @@ lowdiff_status lowdiff_stage_d2h(const void* d_record, uint64_t bytes, void* h_p
  *   st: x (and m = momentum buffer or Adam m, v = Adam v) fp32 device arrays over [lo, hi),
  *     x_bf16 optional device bf16 copy of x written after the last step; st->t, st->adam_step and
  *     st->momentum_initialized are advanced on return (host fields).
+ *     x0/m0/v0: optional full checkpoint C^F_t to load from (Alg.1 line 17, M_t <- Load(C^F_t)):
+ *     when set, the replay reads the starting state from them and writes the result to x/m/v
+ *     (same HBM traffic as in place; the checkpoint stays untouched). NULL = in place.
  * Errors: ECHAIN (t gap/overlap, n/lo/hi/nranks mismatch), ECORRUPT (header), EUNSUPPORTED.
  * ------------------------------------------------------------------------------------------- */
 typedef struct {
@@ -202,6 +205,7 @@ typedef struct {
   uint64_t t;                         /* iteration whose G~ is applied next */
   uint64_t adam_step;                 /* Adam step count stored in the full checkpoint */
   int32_t momentum_initialized;
+  const float* x0; const float* m0; const float* v0;   /* optional source checkpoint (see above) */
 } lowdiff_state;
 
 typedef struct {

@@ -59,7 +59,8 @@ class Opt(C.Structure):
 class State(C.Structure):
     _fields_ = [("x", C.c_void_p), ("m", C.c_void_p), ("v", C.c_void_p), ("x_bf16", C.c_void_p),
                 ("n", C.c_uint64), ("lo", C.c_uint64), ("hi", C.c_uint64), ("t", C.c_uint64),
-                ("adam_step", C.c_uint64), ("momentum_initialized", C.c_int32)]
+                ("adam_step", C.c_uint64), ("momentum_initialized", C.c_int32),
+                ("x0", C.c_void_p), ("m0", C.c_void_p), ("v0", C.c_void_p)]
 
 
 class RecordView(C.Structure):
@@ -407,7 +408,8 @@ def replay(state: dict, opt: dict, records, ws=None, stream=None) -> dict:
             opt.get("eps", 1e-8), int(opt.get("nesterov", 0)), int(opt.get("allow_accumulated_sum", 0)))
     ptr = lambda key: _cuda(state[key], key) if state.get(key) is not None else None
     st = State(ptr("x"), ptr("m"), ptr("v"), ptr("x_bf16"), state["n"], state["lo"], state["hi"],
-               state["t"], state["adam_step"], state["momentum_initialized"])
+               state["t"], state["adam_step"], state["momentum_initialized"],
+               ptr("x0"), ptr("m0"), ptr("v0"))
     R = len(records)
     views = (RecordView * max(R, 1))()
     keep = []

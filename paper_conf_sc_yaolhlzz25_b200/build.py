@@ -60,7 +60,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
     def compile_one(src: str) -> str:
         obj = os.path.join(BUILD, os.path.basename(src) + ".o")
-        cmd = [NVCC, *ARCH, *CFLAGS, *inc, "-c", src, "-o", obj]
+        extra = os.environ.get("LOWDIFF_NVCC_EXTRA", "").split()   # experiments, e.g. -DLOWDIFF_REPLAY_MINB=4
+        cmd = [NVCC, *ARCH, *CFLAGS, *extra, *inc, "-c", src, "-o", obj]
         if verbose:
             print(" ".join(cmd), flush=True)
         r = subprocess.run(cmd, capture_output=True, text=True)

@@ -415,7 +415,8 @@ static lowdiff_status check_state(const lowdiff_state* st, const lowdiff_opt* o)
   if (o->kind != LOWDIFF_OPT_SGD && !st->m) return fail(LOWDIFF_EINVAL, "replay: m required");
   if (o->kind == LOWDIFF_OPT_ADAM && !st->v) return fail(LOWDIFF_EINVAL, "replay: v required");
   if (!aligned16(st->x) || (st->m && !aligned16(st->m)) || (st->v && !aligned16(st->v)) ||
-      (st->x_bf16 && (reinterpret_cast<uintptr_t>(st->x_bf16) & 7u)))
+      (st->x_bf16 && (reinterpret_cast<uintptr_t>(st->x_bf16) & 7u)) ||
+      (st->x0 && !aligned16(st->x0)) || (st->m0 && !aligned16(st->m0)) || (st->v0 && !aligned16(st->v0)))
     return fail(LOWDIFF_EINVAL, "replay: misaligned state");
   return LOWDIFF_OK;
 }
