@@ -309,9 +309,20 @@ __device__ __forceinline__ void select_pass(const float* __restrict__ src, uint6
   constexpr int SH = shift(PASS);
   for (int b = threadIdx.x; b < NB; b += kThreads) sh[b] = 0;
   __syncthreads();
-  for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < N; i += (uint64_t)gridDim.x * kThreads) {
-    const uint32_t key = mag_key(src[i]);
-    if (PASS == 0 || (key >> shift(PASS > 0 ? PASS - 1 : 0)) == prefix) atomicAdd(&sh[(key >> SH) & (NB - 1)], 1u);
+  // Warp-aggregated increments: the candidates' keys crowd into few bins, so lanes with the same
+  // bin are combined (__match_any_sync) into one shared-memory atomic.
+  const int lane = threadIdx.x & 31;
+  const uint64_t stride = (uint64_t)gridDim.x * kThreads;
+  for (uint64_t base = (uint64_t)blockIdx.x * kThreads + (threadIdx.x & ~31u); base < N; base += stride) {
+    const uint64_t i = base + lane;
+    const uint32_t key = i < N ? mag_key(src[i]) : 0u;
+    const bool take = i < N && (PASS == 0 || (key >> shift(PASS > 0 ? PASS - 1 : 0)) == prefix);
+    const uint32_t act = __ballot_sync(0xFFFFFFFFu, take);
+    if (take) {
+      const uint32_t bin = (key >> SH) & (NB - 1);
+      const uint32_t peers = __match_any_sync(act, bin);
+      if (lane == __ffs(peers) - 1) atomicAdd(&sh[bin], (uint32_t)__popc(peers));
+    }
   }
   __syncthreads();
   for (int b = threadIdx.x; b < NB; b += kThreads)
@@ -361,7 +372,7 @@ __device__ __forceinline__ uint64_t block_offset(const uint64_t* bsum, uint64_t*
 }
 
 template <bool VBF16>
-__global__ void __launch_bounds__(kThreads) select_kernel(float* __restrict__ r, uint64_t n, uint64_t k,
+__global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__ r, uint64_t n, uint64_t k,
                                                           Ctl* ctl, const float* __restrict__ cand_val,
                                                           const uint32_t* __restrict__ cand_idx,
                                                           const uint2* __restrict__ tile_info,
@@ -389,10 +400,14 @@ __global__ void __launch_bounds__(kThreads) select_kernel(float* __restrict__ r,
   }
   if (mode != 0) return;                           // full-array fallback: emit_kernel does it
   // ---- candidate mode: fused ordered emission ----
-  // (1) exclusive scan of packed (gt << 32 | eq) flags over the candidate buffer positions
+  // Chunks are powers of two so chunk(p) is a shift. boff: [0,G) block totals, [G,2G) flag-scan
+  // block offsets, [2G,3G) tile-scan block totals.
   const uint32_t G = gridDim.x, b = blockIdx.x;
-  const uint32_t cs = (uint32_t)((N + 1 + G - 1) / G);
-  const uint64_t a0 = (uint64_t)b * cs, a1 = (a0 + cs < N + 1) ? a0 + cs : N + 1;
+  uint32_t cs_log = 0, ts_log = 0;
+  while (((uint64_t)G << cs_log) < N + 1) ++cs_log;
+  while (((uint64_t)G << ts_log) < num_tiles) ++ts_log;
+  // (1) exclusive scan of packed (gt << 32 | eq) flags over the candidate buffer positions
+  const uint64_t a0 = (uint64_t)b << cs_log, a1 = (a0 + (1ull << cs_log) < N + 1) ? a0 + (1ull << cs_log) : N + 1;
   auto flag = [&](uint64_t p) -> uint64_t {
     if (p >= N) return 0;
     const uint32_t key = mag_key(cand_val[p]);
@@ -403,23 +418,27 @@ __global__ void __launch_bounds__(kThreads) select_kernel(float* __restrict__ r,
   grid.sync();
   const uint64_t soff = block_offset(boff, s_scan);
   __syncthreads();
-  if (threadIdx.x == 0) boff[G + b] = soff;        // second half: per-block offsets
+  if (threadIdx.x == 0) boff[G + b] = soff;
   grid.sync();
-  auto S = [&](uint64_t p) -> uint64_t { return sloc[p] + __ldcg(boff + G + (uint32_t)p / cs); };
+  auto S = [&](uint64_t p) -> uint64_t { return sloc[p] + __ldcg(boff + G + (p >> cs_log)); };
   // (2) exclusive scan over tiles (index order) of the per-tile counts S(end) - S(begin)
-  const uint32_t ts = (num_tiles + G - 1) / G;
-  const uint64_t t0 = (uint64_t)b * ts, t1 = (t0 + ts < num_tiles) ? t0 + ts : num_tiles;
+  const uint64_t t0 = (uint64_t)b << ts_log, t1 = (t0 + (1ull << ts_log) < num_tiles) ? t0 + (1ull << ts_log) : num_tiles;
   auto tcount = [&](uint64_t t) -> uint64_t {
     const uint2 ti = tile_info[t];
     return S((uint64_t)ti.x + ti.y) - S(ti.x);
   };
   const uint64_t ttot = t0 < t1 ? chunk_scan(t0, t1, tcount, tloc, s_scan) : 0;
-  grid.sync();                                     // everyone has read boff[b] (first half)
-  if (threadIdx.x == 0) boff[b] = ttot;
+  if (threadIdx.x == 0) boff[2 * G + b] = ttot;
   grid.sync();
-  const uint64_t toff = block_offset(boff, s_scan);
-  __syncthreads();
-  if (threadIdx.x == 0) boff[2 * G + b] = toff;
+  const uint64_t toff = block_offset(boff + 2 * G, s_scan);
+  // (2b) per tile: adjustment = tile prefix - S(segment start), as two int32 fields, so that a
+  //      candidate's (gt_before, eq_before) = S(i) + adj[tile]
+  for (uint64_t t = t0 + threadIdx.x; t < t1; t += kThreads) {
+    const uint64_t tp = tloc[t] + toff;
+    const uint64_t s0 = S(tile_info[t].x);
+    const int32_t dg = (int32_t)((tp >> 32) - (s0 >> 32)), de = (int32_t)((tp & 0xFFFFFFFFull) - (s0 & 0xFFFFFFFFull));
+    tloc[t] = ((uint64_t)(uint32_t)dg << 32) | (uint32_t)de;
+  }
   grid.sync();
   // (3) every candidate finds its output position; selected ones are written (ascending index)
   uint32_t* out_idx = reinterpret_cast<uint32_t*>(pairs);
@@ -430,16 +449,9 @@ __global__ void __launch_bounds__(kThreads) select_kernel(float* __restrict__ r,
     const uint64_t vp = pad16(4 * k) + (VBF16 ? 2 : 4) * k, ve = pad16(4 * k) + pad16((VBF16 ? 2 : 4) * k);
     if (vp + threadIdx.x < ve) pairs[vp + threadIdx.x] = 0;
   }
-  for (uint64_t i = (uint64_t)b * kThreads + threadIdx.x; i < N; i += (uint64_t)G * kThreads) {
-    const float a = cand_val[i];
-    const uint32_t key = mag_key(a);
-    if (key < K) continue;
-    const uint32_t idx = cand_idx[i];
-    const uint32_t t = idx / kTile;
-    const uint64_t tp = tloc[t] + __ldcg(boff + 2 * G + t / ts);
-    const uint64_t in_tile = S(i) - S(tile_info[t].x);
-    const uint64_t gtb = (tp >> 32) + (in_tile >> 32);
-    const uint64_t eqb = (tp & 0xFFFFFFFFull) + (in_tile & 0xFFFFFFFFull);
+  auto emit = [&](uint64_t i, float a, uint32_t key, uint32_t idx, uint64_t si, uint64_t adj) {
+    const uint64_t gtb = (uint64_t)((int64_t)(si >> 32) + (int32_t)(adj >> 32));
+    const uint64_t eqb = (uint64_t)((int64_t)(si & 0xFFFFFFFFull) + (int32_t)(uint32_t)adj);
     if (key > K || eqb < m) {
       const uint64_t pos = gtb + (eqb < m ? eqb : m);
       out_idx[pos] = idx;
@@ -452,6 +464,22 @@ __global__ void __launch_bounds__(kThreads) select_kernel(float* __restrict__ r,
         r[idx] = 0.0f;
       }
     }
+  };
+  const uint64_t stride = (uint64_t)G * kThreads;
+  for (uint64_t i0 = (uint64_t)b * kThreads + threadIdx.x; i0 < N; i0 += 2 * stride) {
+    // two candidates per round, their independent loads issued together
+    const uint64_t i1 = i0 + stride;
+    const bool has1 = i1 < N;
+    const float a0v = cand_val[i0], a1v = has1 ? cand_val[i1] : 0.f;
+    const uint32_t k0 = mag_key(a0v), k1 = has1 ? mag_key(a1v) : 0u;
+    const bool s0 = k0 >= K, s1 = has1 && k1 >= K;
+    uint32_t x0 = 0, x1 = 0;
+    uint64_t S0 = 0, S1 = 0;
+    if (s0) { x0 = cand_idx[i0]; S0 = S(i0); }
+    if (s1) { x1 = cand_idx[i1]; S1 = S(i1); }
+    const uint64_t adj0 = s0 ? tloc[x0 / kTile] : 0, adj1 = s1 ? tloc[x1 / kTile] : 0;
+    if (s0) emit(i0, a0v, k0, x0, S0, adj0);
+    if (s1) emit(i1, a1v, k1, x1, S1, adj1);
   }
 }
 
@@ -626,9 +654,10 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   Ctl* ctl = reinterpret_cast<Ctl*>(w + L.ctl);
   LD_CUDA(cudaMemsetAsync(w, 0, L.zero_end, s), "memset compress workspace");
 
-  // sample size: >= 2048 expected keys above the k-th (S >= 2048 n / k), >= 64 Ki, power of 2
+  // sample size: >= 1024 expected keys above the k-th (S >= 1024 n / k: the 1.3x target is then
+  // ~9 sigma above k), >= 64 Ki, power of 2
   uint64_t S = 65536;
-  while ((double)S * (double)k < 2048.0 * (double)n && S < (1ull << 26)) S <<= 1;
+  while ((double)S * (double)k < 1024.0 * (double)n && S < (1ull << 26)) S <<= 1;
   const int exhaustive = (S >= n / 2) ? 1 : 0;
   const uint32_t micro = exhaustive ? (uint32_t)((n + 7) / 8) : (uint32_t)(S / 8);
   const double stride = exhaustive ? 1.0 : (double)(n / 8) / (double)micro;
@@ -659,15 +688,22 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
               L.num_tiles, ctl, tiles, cidx, cval, L.cap);
 
   {
-    static int sel_grid = 0;
-    if (!sel_grid) {
-      int per_sm = 0;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, select_kernel<false>, kThreads, 0);
-      int per_sm2 = 0;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm2, select_kernel<true>, kThreads, 0);
-      if (per_sm2 < per_sm) per_sm = per_sm2;
-      sel_grid = (per_sm >= 2 ? 2 : 1) * kNumSMs;
+    static int sel_max = 0;                        // occupancy limit (CTAs per SM), both variants
+    if (!sel_max) {
+      int a = 0, b2 = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, select_kernel<false>, kThreads, 0);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b2, select_kernel<true>, kThreads, 0);
+      sel_max = a < b2 ? a : b2;
+      if (sel_max < 1) sel_max = 1;
+      if (sel_max > kMaxSelectBlocks / kNumSMs) sel_max = kMaxSelectBlocks / kNumSMs;
     }
+    // CTAs per SM: more hide the latency of the emission loop at large k, fewer make the grid
+    // syncs and histogram flushes cheaper at small k (measured, profiles/README.md).
+    int want = k >= (1u << 18) ? 4 : 2;
+    if (const char* e = getenv("LOWDIFF_SELECT_PER_SM")) want = atoi(e);
+    if (want < 1) want = 1;
+    if (want > sel_max) want = sel_max;
+    const int sel_grid = want * kNumSMs;
     float* rr = residual;
     uint32_t *h0 = reinterpret_cast<uint32_t*>(w + L.h0), *h1 = reinterpret_cast<uint32_t*>(w + L.h1),
              *h2 = reinterpret_cast<uint32_t*>(w + L.h2);

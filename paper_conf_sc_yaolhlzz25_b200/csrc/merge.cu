@@ -603,13 +603,14 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
   LD_LAUNCH("starts", s, starts_kernel<kW>, dim3((unsigned)gx, (unsigned)ls.L), kThreads, 0, ls, lo, hi,
             M.num_w, starts);
 
-  // group size: about kCap/2 entries per group at the average density (power of two)
+  // group size: up to kCap/2 entries per group at the average density (power of two); the
+  // entries actually present (max_entries is a capacity) make groups smaller than this bound
   const double per_w = (double)max_entries / (double)M.num_w;
   uint32_t G = 1;
   while (G < 4096 && (double)(2 * G) * per_w <= kCap / 2) G <<= 1;     // key < 2^24
   LD_LAUNCH("merge_plan", s, plan_kernel, 1, kPlanThreads, 0, ls.L, starts, M.num_w, G, ctl, items);
 
-  const int grid = (int)(M.num_w < 3u * kNumSMs ? M.num_w : 3u * kNumSMs);
+  const int grid = (int)(M.num_w < 6u * kNumSMs ? M.num_w : 6u * kNumSMs);   // 6 CTAs/SM (37 KB smem)
   uint32_t* ucnt = reinterpret_cast<uint32_t*>(w + M.ucnt);
   uint32_t* epre = reinterpret_cast<uint32_t*>(w + M.epre);
   uint32_t* upre = reinterpret_cast<uint32_t*>(w + M.upre);
