@@ -2,17 +2,18 @@
 """LowDiff hot-path benchmark (BASELINE.json metric: "diff-build & replay gradient GB/s at
 1/2/4/8 B200, % of HBM roofline").
 
-One STEP = one pass of the whole hot path over one batch:
-  for each of the B iterations of the batch: compress (top-k + EF) -> sparse all-gather (NCCL for
-  P > 1) + coalesce of this rank's shard -> ring slot;
-  then batch merge of the B differentials (STACK, Adam) -> record -> async D2H stage into pinned
-  host memory (copy stream) -> replay of the record onto this rank's full-checkpoint shard.
-value = gradient bytes all ranks fed through the path per second = P * B * n * sizeof(g) / t_step.
+One STEP = one pass of the whole hot path over one replay chain of
+K = R*B iterations (the config's chain length; R = K/B batch records):
+  R times: B iterations of compress (top-k + EF) -> sparse all-gather (NCCL for P > 1) + coalesce
+  of this rank's shard -> ring slot; then batch merge of the B differentials -> record -> async
+  D2H stage into pinned host memory (copy stream);
+  then recovery: Load(C^F) + replay of the R-record chain onto this rank's checkpoint shard.
+value = gradient bytes all ranks fed through the path per second = P * K * n * sizeof(g) / t_step.
 
 Workload (N = 1 line): config C3 = BASELINE configs[2], the VGG-16-shaped gradient the metric's
-1/2/4/8-GPU scaling is quoted on (n = 138,357,544 fp32, rho = 0.001, B = 16, Adam replay of the
-batch's 16 iterations). Inputs are synthetic (workloads/, seeded), resident in HBM before timing;
-every gradient (553 MB) is larger than the 126 MB L2, so no flush is needed between steps.
+1/2/4/8-GPU scaling is quoted on (n = 138,357,544 fp32, rho = 0.001, B = 16, K = 16: one record,
+Adam replay of its 16 iterations). Inputs are synthetic (workloads/, seeded), resident in HBM
+before timing; every gradient (553 MB) is larger than the 126 MB L2, so no flush is needed.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--config 3] [--impl ours|reference]
   torchrun --nproc-per-node N bench.py --gpus N ...
@@ -56,34 +57,42 @@ def parse_args():
 # ---------------------------------------------------------------------------------------------
 def oracle_step_sample(cfg, n_s: int, t0: int = 0):
     """Time the oracle on one step of the same workload restricted to the first n_s gradient
-    elements (same rho, B, optimizer): B compress + coalesce, one merge, one replay. Returns
-    (seconds, gradient bytes processed)."""
+    elements (same rho, B, chain length, optimizer): R = K/B batches of B compress + coalesce and
+    one merge each, then one replay of the R-record chain. Returns (seconds, gradient bytes)."""
     import numpy as np
     import oracle
     from workloads import gradient, segment_sigmas
+    import torch
     sig = segment_sigmas(cfg)[:n_s]
     k = max(1, int(cfg.rho * n_s))
+    R = chain_records(cfg)
     grads = [gradient(cfg, 0, t0 + t, "cpu", sigmas=sig, n=n_s) for t in range(cfg.B)]
-    grads = [g.view(np.int16).numpy().view(np.uint16) if cfg.gdt == "bf16" else g.numpy() for g in
-             [gg.view(__import__("torch").int16) if cfg.gdt == "bf16" else gg for gg in grads]]
+    grads = [g.view(torch.int16).numpy().view(np.uint16) if cfg.gdt == "bf16" else g.numpy() for g in grads]
     r = np.zeros(n_s, np.float32)
     lr = np.float32(cfg.hyper["lr"])
     x = np.zeros(n_s, np.float32); m = np.zeros(n_s, np.float32); v = np.zeros(n_s, np.float32)
     o_vdt = oracle.BF16 if cfg.vdt == "bf16" else oracle.F32
-    t_start = time.perf_counter()
-    diffs = []
-    for t in range(cfg.B):
-        idx, val, r = oracle.compress(grads[t], r, k, o_vdt)
-        diffs.append(oracle.coalesce([oracle.pairs_pack(idx, val, o_vdt)], k, o_vdt, 0, n_s, True))
     mode = oracle.STACK if cfg.merge == "stack" else oracle.SUM
-    rec = oracle.batch_merge(diffs, lr, mode, n_s, 0, n_s, t0, 1)
+    t_start = time.perf_counter()
+    recs = []
+    for b in range(R):
+        diffs = []
+        for t in range(cfg.B):
+            idx, val, r = oracle.compress(grads[t], r, k, o_vdt)
+            diffs.append(oracle.coalesce([oracle.pairs_pack(idx, val, o_vdt)], k, o_vdt, 0, n_s, True))
+        recs.append(oracle.batch_merge(diffs, lr, mode, n_s, 0, n_s, t0 + b * cfg.B, 1))
     st = {"x": x, "m": m if cfg.opt != "sgd" else None, "v": v if cfg.opt == "adam" else None,
           "n": n_s, "lo": 0, "hi": n_s, "t": t0, "adam_step": 1000, "momentum_initialized": 1}
     opt = {"kind": cfg.opt, **{k2: v2 for k2, v2 in cfg.hyper.items() if k2 != "lr"}}
-    oracle.replay(opt, st, [rec])
+    oracle.replay(opt, st, recs)
     dt = time.perf_counter() - t_start
-    gbytes = cfg.B * n_s * (2 if cfg.gdt == "bf16" else 4)
+    gbytes = R * cfg.B * n_s * (2 if cfg.gdt == "bf16" else 4)
     return dt, gbytes
+
+
+def chain_records(cfg) -> int:
+    """Records per step: the config's replay chain of K differentials is K/B batch records."""
+    return max(1, cfg.K // cfg.B)
 
 
 def run_reference(args, cfg):
@@ -100,13 +109,14 @@ def run_reference(args, cfg):
     tot = sum(times)
     val = args.steps * gb / tot / 1e9
     sample = (f"oracle (plain C++, 1 thread) full step of {cfg.name} on the first {n_s} of n={cfg.n} "
-              f"gradient elements (rho={cfg.rho}, B={cfg.B}, {cfg.opt} replay)")
+              f"gradient elements (rho={cfg.rho}, {chain_records(cfg)} batches of B={cfg.B}, {cfg.opt} replay "
+              f"of the {cfg.K}-iteration chain)")
     line = {"impl": "reference", "metric": "diff-build & replay gradient GB/s at 1/2/4/8 B200, % of HBM roofline",
             "value": val, "unit": "GB/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1e3 * tot / args.steps, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f32" if cfg.gdt == "f32" else "bf16", "data": "synthetic",
             "config": {"workload": cfg.name, "n": cfg.n, "n_sample": n_s, "rho": cfg.rho, "B": cfg.B,
-                       "replay": cfg.opt},
+                       "replay": f"{cfg.opt}, chain of {cfg.K} iterations ({chain_records(cfg)} records)"},
             "cpu_baseline": {"value": val, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample},
             "e2e": {"value": val, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -203,10 +213,11 @@ def run_ours(args, cfg):
              torch.zeros(1, dtype=torch.int64, device=dev)) for _ in range(B)]
     pairs = torch.empty(ld.pairs_bytes(k, cfg.vdt), dtype=torch.uint8, device=dev)
     rec_cap = ld.record_max_bytes(cfg.merge, B, B * cap)
-    record = torch.empty(rec_cap, dtype=torch.uint8, device=dev)
+    R = chain_records(cfg)                              # batch records per step (replay chain K = R*B)
+    records = [torch.empty(rec_cap, dtype=torch.uint8, device=dev) for _ in range(R)]
     d_bytes = torch.zeros(1, dtype=torch.int64, device=dev)
-    head = torch.empty(80 + 4 * B + 16, dtype=torch.uint8, pin_memory=True)
-    staged = torch.empty(rec_cap, dtype=torch.uint8, pin_memory=True)
+    heads = [torch.empty(80 + 4 * B + 16, dtype=torch.uint8, pin_memory=True) for _ in range(R)]
+    staged = [torch.empty(rec_cap, dtype=torch.uint8, pin_memory=True) for _ in range(R)]
     main = torch.cuda.current_stream()
     copy_stream = torch.cuda.Stream()
     t_iter = [0]
@@ -222,30 +233,37 @@ def run_ours(args, cfg):
             ld.compress(g, r, k, vdt=cfg.vdt, pairs=pairs)
             ld.allgather_sparse(comm, pairs, k, cfg.vdt, lo, hi, True, *ring[j])
 
-    def checkpoint_phase():
-        """Batch merge -> record -> D2H stage (copy stream) -> replay of the record; returns bytes."""
+    def checkpoint_phase(b):
+        """Batch merge -> record b -> async D2H stage (copy stream); returns the record's bytes."""
         diffs = [(ring[j][0], ring[j][1], ring[j][2], cap, lr) for j in range(B)]
-        ld.batch_merge(diffs, cfg.merge, n, lo, hi, t_iter[0], P, record=record, d_record_bytes=d_bytes)
+        ld.batch_merge(diffs, cfg.merge, n, lo, hi, t_iter[0], P, record=records[b], d_record_bytes=d_bytes)
         nb = ld.record_bytes(d_bytes, rec_cap)          # the checkpoint thread's only sync
-        ld.stage_d2h(record, 80 + 4 * B, head, main)    # header + lr[] for the host-side replay call
+        ld.stage_d2h(records[b], 80 + 4 * B, heads[b], main)   # header + lr[] for the host-side replay
         copy_stream.wait_stream(main)
-        ld.stage_d2h(record, nb, staged, copy_stream)   # async persist staging (copy engine)
-        main.synchronize()
-        state["t"] = t_iter[0]                          # the checkpoint is stamped at this batch's start
-        state["adam_step"] = ck["adam_step"]
-        state["momentum_initialized"] = ck["momentum_initialized"]
-        ld.replay(state, opt, [(record, head)])
-        main.wait_stream(copy_stream)
+        ld.stage_d2h(records[b], nb, staged[b], copy_stream)   # async persist staging (copy engine)
         t_iter[0] += B
         return nb
 
+    def recovery_phase():
+        """Load(C^F) + replay of the step's chain of R records (K = R*B iterations)."""
+        main.synchronize()                              # the replay call reads the staged headers
+        state["t"] = t_iter[0] - R * B                  # the checkpoint is stamped at the chain start
+        state["adam_step"] = ck["adam_step"]
+        state["momentum_initialized"] = ck["momentum_initialized"]
+        ld.replay(state, opt, [(records[b], heads[b]) for b in range(R)])
+        main.wait_stream(copy_stream)
+
     def step(graph=None, h2d=None):
-        """One pass of the path over one batch."""
-        if graph is not None:
-            graph.replay()
-        else:
-            build_phase(h2d)
-        return checkpoint_phase()
+        """One pass of the path: R batches built, merged and staged, then the chain replayed."""
+        nb = 0
+        for b in range(R):
+            if graph is not None:
+                graph.replay()
+            else:
+                build_phase(h2d)
+            nb += checkpoint_phase(b)
+        recovery_phase()
+        return nb
 
     def timed(nsteps, **kw):
         if world > 1:
@@ -302,10 +320,10 @@ def run_ours(args, cfg):
     pms, _ = timed(args.steps)
     ld.profile_enable(False)
     prof = {c: ld.profile_query(c) for c in ("compress_stream", "compress_sample", "compress_select",
-                                             "compress_emit", "coalesce", "starts", "merge", "merge_pack",
+                                             "coalesce", "starts", "merge", "merge_pack",
                                              "replay_dense", "replay_sparse")}
     ms_step = ms / args.steps
-    value = P * B * n * gsz / (ms_step * 1e-3) / 1e9
+    value = P * R * B * n * gsz / (ms_step * 1e-3) / 1e9
 
     # ---- roofline of the dominant kernel (measured live over the timed region) ----
     peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
@@ -346,8 +364,8 @@ def run_ours(args, cfg):
         e_steps = max(1, min(args.steps, 3))
         ems, enb = timed(e_steps, **kw)
         e_ms = ems / e_steps
-        e2e = {"value": P * B * n * gsz / (e_ms * 1e-3) / 1e9, "unit": "GB/s",
-               "h2d_bytes_per_step": B * n * gsz, "d2h_bytes_per_step": int(enb) + 80 + 4 * B + 8,
+        e2e = {"value": P * R * B * n * gsz / (e_ms * 1e-3) / 1e9, "unit": "GB/s",
+               "h2d_bytes_per_step": R * B * n * gsz, "d2h_bytes_per_step": int(enb) + R * (80 + 4 * B + 8),
                "ms_per_step": e_ms, "steps": e_steps}
 
     # ---- CPU oracle baseline (rank 0, N = 1 only) ----
@@ -365,13 +383,14 @@ def run_ours(args, cfg):
                 "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
                 "dtype": "f32" if cfg.gdt == "f32" else "bf16", "data": "synthetic",
                 "config": {"workload": cfg.name, "n": n, "k": k, "rho": cfg.rho, "B": B, "P": P,
-                           "shard": [lo, hi], "replay": f"{cfg.opt}, {B} iterations (1 {cfg.merge.upper()} record)",
+                           "shard": [lo, hi], "replay": f"{cfg.opt}, chain of {R * B} iterations ({R} {cfg.merge.upper()} record{'s' if R > 1 else ''} of B={B})",
                            "l2": (f"inputs larger than L2 (each gradient {n * gsz / 1e6:.0f} MB > 126 MB), no flush"
                                   if n * gsz > 126e6 else
                                   f"working set {n * (gsz + 8) / 1e6:.1f} MB fits L2 (latency-class config)"),
                            "grad_pool": pool,
-                           "differentials_per_s": P * B / (ms_step * 1e-3),
-                           "replayed_iterations_per_s": B / (ms_step * 1e-3),
+                           "batches_per_step": R,
+                           "differentials_per_s": P * R * B / (ms_step * 1e-3),
+                           "replayed_iterations_per_s": R * B / (ms_step * 1e-3),
                            "record_bytes": int(rec_bytes)},
                 "timing": {"build_phase": "one CUDA graph per step" if graph is not None else "eager launches",
                            "profiled_ms_per_step": pms / args.steps,

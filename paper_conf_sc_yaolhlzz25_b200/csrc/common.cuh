@@ -16,15 +16,7 @@ __host__ __device__ inline uint64_t pad16(uint64_t x) { return (x + 15u) & ~(uin
 // |a| as an ordered u32 key: sign dropped, so +0 == -0 (reading #3).
 __device__ __forceinline__ uint32_t mag_key(float a) { return __float_as_uint(a) & 0x7FFFFFFFu; }
 
-// ---- memory-order helpers (decoupled look-back) ------------------------------------------
-__device__ __forceinline__ void st_release(uint64_t* p, uint64_t v) {
-  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ uint64_t ld_acquire(const uint64_t* p) {
-  uint64_t v;
-  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
+// ---- streaming loads ---------------------------------------------------------------------
 __device__ __forceinline__ float4 ld_stream_f4(const float4* p) {   // read once: no L1 allocate
   float4 r;
   asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
@@ -37,41 +29,6 @@ __device__ __forceinline__ uint2 ld_stream_u2(const uint2* p) {
   return r;
 }
 
-// Decoupled look-back (single-pass prefix scan over tiles processed in ticket order).
-// status[t] = (flag << 62) | value; flag 1 = tile aggregate, 2 = inclusive prefix.
-// Called by ONE full warp; returns the exclusive prefix of `aggregate` over tiles < tile and
-// publishes the inclusive prefix. Values must stay below 2^62.
-constexpr uint64_t kLbMask = (1ull << 62) - 1;
-__device__ inline uint64_t lookback_exclusive(uint64_t* status, uint32_t tile, uint64_t aggregate) {
-  const int lane = threadIdx.x & 31;
-  if (tile == 0) {
-    if (lane == 0) st_release(status, (2ull << 62) | aggregate);
-    return 0;
-  }
-  if (lane == 0) st_release(status + tile, (1ull << 62) | aggregate);
-  uint64_t exclusive = 0;
-  int64_t base = (int64_t)tile - 1;
-  while (true) {
-    const int64_t my = base - lane;
-    uint64_t w;
-    do {
-      w = (my >= 0) ? ld_acquire(status + my) : (2ull << 62);
-    } while (__any_sync(0xFFFFFFFFu, (w >> 62) == 0));
-    const uint32_t incl = __ballot_sync(0xFFFFFFFFu, (w >> 62) == 2);
-    uint64_t v = w & kLbMask;
-    if (incl) {
-      const int first = __ffs(incl) - 1;            // nearest predecessor holding a prefix
-      if (lane > first) v = 0;
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, o);
-    exclusive += v;
-    if (incl) break;
-    base -= 32;
-  }
-  if (lane == 0) st_release(status + tile, (2ull << 62) | (exclusive + aggregate));
-  return exclusive;
-}
 
 // Block-wide exclusive scan of a u64 (kThreads threads). `smem` holds >= kThreads/32 u64.
 // Returns the exclusive prefix; *total receives the block total. Contains two __syncthreads.

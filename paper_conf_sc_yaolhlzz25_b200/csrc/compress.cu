@@ -4,13 +4,14 @@
 // Design: the only HBM-heavy step is one fused streaming pass
 //   a = g + r;  r <- a;  if |a| >= T_est: append (i, a) to a candidate buffer
 // which moves the algorithmic floor of 12n bytes (fp32 g) / 10n (bf16 g). T_est comes from a
-// small stratified sample of |g + r| (1/rho-scaled, contiguous 4 KB chunks) so the candidates
-// number ~1.2-2.5 k. An exact 3-digit radix select (12/10/9 bits of the 31-bit key) over the
-// candidates finds the k-th key K* and the number m of K*-ties to keep; an ordered emission pass
-// (decoupled look-back over tiles) writes the k pairs in ascending index order and fixes r on S.
-// If the sample under- or over-shot (candidates < k or > capacity) the select/emit kernels run
-// over the full residual array instead (exact, ~+20n bytes; never observed on the synthetic
-// workloads). Nothing on this path is a dense contraction: no tensor cores.
+// small stratified sample of |g + r| (8-element micro-chunks, >= 1024 n/k of them) so the
+// candidates number ~1.3-2 k. One cooperative kernel then does the rest: an exact 3-digit radix
+// select (12/10/9 bits of the 31-bit key) over the candidates finds the k-th key K* and the number
+// m of K*-ties to keep, and an ordered emission (per-tile counts, a scan over tiles, ballot
+// prefixes inside each tile) writes the k pairs in ascending index order and fixes r on S.
+// If the sample under- or over-shot (candidates < k or > capacity) the same kernel runs over the
+// full residual array instead (exact, ~+12n bytes; not observed on the synthetic workloads).
+// Nothing on this path is a dense contraction: no tensor cores.
 #include <stdio.h>
 
 #include <cooperative_groups.h>
@@ -24,7 +25,6 @@ namespace lowdiff {
 namespace {
 
 constexpr int kTile = 4096;            // elements per streaming tile: 256 thr x 4 vectors x 4
-constexpr int kTilesPerEmit = kThreads; // streaming tiles per emission block (one per thread)
 constexpr int kMaxSelectBlocks = 4 * 148;
 // digit p = (key >> shift(p)) & (bins(p) - 1): 12 + 10 + 9 bits of the 31-bit key
 __host__ __device__ constexpr int bins(int p) { return p == 0 ? 4096 : (p == 1 ? 1024 : 512); }
@@ -38,21 +38,20 @@ struct __align__(256) Ctl {
   uint32_t sel_ticket[3];
   uint32_t prefix;         // key bits above the current digit
   uint32_t kstar;          // the k-th largest key
-  uint32_t emit_ticket;
+  uint32_t pad0;
   uint64_t k_rem;          // rank still to find below the prefix
   uint64_t count_gt;       // elements with key above the prefix range
   uint64_t m;              // K*-ties to keep (lowest indices first)
 };
 
 struct Layout {
-  uint64_t ctl, hs, h0, h1, h2, status, zero_end, tiles, cand_idx, cand_val, sloc, tloc, boff, total;
-  uint32_t num_tiles, num_emit, cap;
+  uint64_t ctl, hs, h0, h1, h2, zero_end, tiles, cand_idx, cand_val, tloc, boff, total;
+  uint32_t num_tiles, cap;
 };
 
 Layout layout(uint64_t n, uint64_t k) {
   Layout L;
   L.num_tiles = (uint32_t)((n + kTile - 1) / kTile);
-  L.num_emit = (L.num_tiles + kTilesPerEmit - 1) / kTilesPerEmit;
   uint64_t cap = 8 * k + 65536;
   L.cap = (uint32_t)(cap < n ? cap : n);
   uint64_t o = 0;
@@ -61,13 +60,11 @@ Layout layout(uint64_t n, uint64_t k) {
   L.h0 = o;       o += align256(4u * bins(0));
   L.h1 = o;       o += align256(4u * bins(1));
   L.h2 = o;       o += align256(4u * bins(2));
-  L.status = o;   o += align256(8ull * L.num_emit);
   L.zero_end = o;
   L.tiles = o;    o += align256(8ull * L.num_tiles);
   L.cand_idx = o; o += align256(4ull * L.cap);
   L.cand_val = o; o += align256(4ull * L.cap);
-  L.sloc = o;     o += align256(8ull * (L.cap + 1));   // candidate flag scan
-  L.tloc = o;     o += align256(8ull * L.num_tiles);   // tile count scan
+  L.tloc = o;     o += align256(8ull * L.num_tiles);   // per-tile (gt, eq) counts, then their scan
   L.boff = o;     o += align256(8ull * 3 * kMaxSelectBlocks);
   L.total = o;
   return L;
@@ -364,8 +361,15 @@ __device__ __forceinline__ uint64_t chunk_scan(uint64_t a, uint64_t e, ValueFn v
 
 // Exclusive prefix of the blocks' chunk totals (each block sums bsum[0, blockIdx.x)).
 __device__ __forceinline__ uint64_t block_offset(const uint64_t* bsum, uint64_t* s_scan) {
+  uint64_t v[kMaxSelectBlocks / kThreads + 1];     // independent loads, issued together
+#pragma unroll
+  for (int q = 0; q < kMaxSelectBlocks / kThreads + 1; ++q) {
+    const uint32_t b = threadIdx.x + q * kThreads;
+    v[q] = b < blockIdx.x ? __ldcg(bsum + b) : 0;
+  }
   uint64_t part = 0;
-  for (uint32_t b = threadIdx.x; b < blockIdx.x; b += kThreads) part += __ldcg(bsum + b);
+#pragma unroll
+  for (int q = 0; q < kMaxSelectBlocks / kThreads + 1; ++q) part += v[q];
   uint64_t tot;
   block_exclusive_scan(part, s_scan, &tot);
   return tot;
@@ -377,7 +381,7 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
                                                           const uint32_t* __restrict__ cand_idx,
                                                           const uint2* __restrict__ tile_info,
                                                           uint32_t num_tiles, uint32_t cap, uint32_t* h0,
-                                                          uint32_t* h1, uint32_t* h2, uint64_t* sloc,
+                                                          uint32_t* h1, uint32_t* h2,
                                                           uint64_t* tloc, uint64_t* boff, uint8_t* pairs) {
   cg::grid_group grid = cg::this_grid();
   __shared__ uint32_t sh[bins(0)];
@@ -398,49 +402,58 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
     ctl->kstar = K;
     ctl->m = m;
   }
-  if (mode != 0) return;                           // full-array fallback: emit_kernel does it
-  // ---- candidate mode: fused ordered emission ----
-  // Chunks are powers of two so chunk(p) is a shift. boff: [0,G) block totals, [G,2G) flag-scan
-  // block offsets, [2G,3G) tile-scan block totals.
-  const uint32_t G = gridDim.x, b = blockIdx.x;
-  uint32_t cs_log = 0, ts_log = 0;
-  while (((uint64_t)G << cs_log) < N + 1) ++cs_log;
+  // ---- fused ordered emission ----
+  // A streaming tile's candidates sit contiguously in the buffer, in index order (candidate mode),
+  // or the tile is its own 4096 residual elements (full mode, the fallback). A group of g lanes
+  // (a power of two covering the mean segment length, 4..32) owns one tile at a time:
+  //  (A) per tile: (count > K*, count == K*) over its segment -> tcnt[t]
+  //  (B) exclusive scan of tcnt over tiles (block chunks + block offsets)
+  //  (C) per tile again: ballot prefixes inside the segment give each kept candidate its slot
+  // output position of a kept candidate = (# > K* before it) + min(# == K* before it, m).
+  const uint32_t G = gridDim.x, b = blockIdx.x, lane = threadIdx.x & 31;
+  uint32_t ts_log = 0;
   while (((uint64_t)G << ts_log) < num_tiles) ++ts_log;
-  // (1) exclusive scan of packed (gt << 32 | eq) flags over the candidate buffer positions
-  const uint64_t a0 = (uint64_t)b << cs_log, a1 = (a0 + (1ull << cs_log) < N + 1) ? a0 + (1ull << cs_log) : N + 1;
-  auto flag = [&](uint64_t p) -> uint64_t {
-    if (p >= N) return 0;
-    const uint32_t key = mag_key(cand_val[p]);
-    return ((uint64_t)(key > K) << 32) | (uint64_t)(key == K);
+  uint32_t glog = 2;
+  while (glog < 5 && ((uint64_t)num_tiles << glog) < N) ++glog;
+  const float* vsrc = mode ? r : cand_val;
+  auto segment = [&](uint64_t t) -> uint2 {      // (first buffer position, length) of tile t
+    if (mode == 0) return tile_info[t];
+    const uint64_t b0 = t * kTile;
+    return make_uint2((uint32_t)b0, (uint32_t)((n - b0) < (uint64_t)kTile ? n - b0 : kTile));
   };
-  const uint64_t stot = a0 < a1 ? chunk_scan(a0, a1, flag, sloc, s_scan) : 0;
-  if (threadIdx.x == 0) boff[b] = stot;
-  grid.sync();
-  const uint64_t soff = block_offset(boff, s_scan);
-  __syncthreads();
-  if (threadIdx.x == 0) boff[G + b] = soff;
-  grid.sync();
-  auto S = [&](uint64_t p) -> uint64_t { return sloc[p] + __ldcg(boff + G + (p >> cs_log)); };
-  // (2) exclusive scan over tiles (index order) of the per-tile counts S(end) - S(begin)
-  const uint64_t t0 = (uint64_t)b << ts_log, t1 = (t0 + (1ull << ts_log) < num_tiles) ? t0 + (1ull << ts_log) : num_tiles;
-  auto tcount = [&](uint64_t t) -> uint64_t {
-    const uint2 ti = tile_info[t];
-    return S((uint64_t)ti.x + ti.y) - S(ti.x);
-  };
-  const uint64_t ttot = t0 < t1 ? chunk_scan(t0, t1, tcount, tloc, s_scan) : 0;
-  if (threadIdx.x == 0) boff[2 * G + b] = ttot;
-  grid.sync();
-  const uint64_t toff = block_offset(boff + 2 * G, s_scan);
-  // (2b) per tile: adjustment = tile prefix - S(segment start), as two int32 fields, so that a
-  //      candidate's (gt_before, eq_before) = S(i) + adj[tile]
-  for (uint64_t t = t0 + threadIdx.x; t < t1; t += kThreads) {
-    const uint64_t tp = tloc[t] + toff;
-    const uint64_t s0 = S(tile_info[t].x);
-    const int32_t dg = (int32_t)((tp >> 32) - (s0 >> 32)), de = (int32_t)((tp & 0xFFFFFFFFull) - (s0 & 0xFFFFFFFFull));
-    tloc[t] = ((uint64_t)(uint32_t)dg << 32) | (uint32_t)de;
+  const uint32_t g = 1u << glog, gl = lane & (g - 1), gshift = lane & ~(g - 1);
+  const uint32_t gmask = g == 32 ? 0xFFFFFFFFu : ((1u << g) - 1);
+  const uint64_t tpw = 32u >> glog;                // tiles per warp per round
+  const uint64_t wstride = (uint64_t)G * (kThreads / 32) * tpw;
+  const uint64_t tfirst = (((uint64_t)b * kThreads + threadIdx.x) >> 5) * tpw + (lane >> glog);
+  uint64_t* tcnt = tloc;
+  // (A)
+  for (uint64_t tw = tfirst - (lane >> glog); tw < num_tiles; tw += wstride) {   // warp-uniform
+    const uint64_t t = tw + (lane >> glog);
+    const uint2 ti = t < num_tiles ? segment(t) : make_uint2(0u, 0u);
+    uint32_t gt = 0, eq = 0;
+    for (uint32_t j = gl; j < ti.y; j += g) {
+      const uint32_t key = mag_key(vsrc[(uint64_t)ti.x + j]);
+      gt += key > K;
+      eq += key == K;
+    }
+    for (uint32_t o = g >> 1; o; o >>= 1) {        // reduce inside the group
+      gt += __shfl_xor_sync(0xFFFFFFFFu, gt, o);
+      eq += __shfl_xor_sync(0xFFFFFFFFu, eq, o);
+    }
+    if (gl == 0 && t < num_tiles) tcnt[t] = ((uint64_t)gt << 32) | eq;
   }
   grid.sync();
-  // (3) every candidate finds its output position; selected ones are written (ascending index)
+  // (B)
+  const uint64_t t0 = (uint64_t)b << ts_log, t1 = (t0 + (1ull << ts_log) < num_tiles) ? t0 + (1ull << ts_log) : num_tiles;
+  const uint64_t ttot = t0 < t1 ? chunk_scan(t0, t1, [&](uint64_t t) { return tcnt[t]; }, tcnt, s_scan) : 0;
+  if (threadIdx.x == 0) boff[b] = ttot;
+  grid.sync();
+  const uint64_t toff = block_offset(boff, s_scan);
+  __syncthreads();
+  if (threadIdx.x == 0) boff[G + b] = toff;
+  grid.sync();
+  // (C)
   uint32_t* out_idx = reinterpret_cast<uint32_t*>(pairs);
   uint8_t* out_val = pairs + pad16(4 * k);
   if (b == 0 && threadIdx.x < 16) {                // zero the 16-byte padding of both sections
@@ -449,168 +462,43 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
     const uint64_t vp = pad16(4 * k) + (VBF16 ? 2 : 4) * k, ve = pad16(4 * k) + pad16((VBF16 ? 2 : 4) * k);
     if (vp + threadIdx.x < ve) pairs[vp + threadIdx.x] = 0;
   }
-  auto emit = [&](uint64_t i, float a, uint32_t key, uint32_t idx, uint64_t si, uint64_t adj) {
-    const uint64_t gtb = (uint64_t)((int64_t)(si >> 32) + (int32_t)(adj >> 32));
-    const uint64_t eqb = (uint64_t)((int64_t)(si & 0xFFFFFFFFull) + (int32_t)(uint32_t)adj);
-    if (key > K || eqb < m) {
-      const uint64_t pos = gtb + (eqb < m ? eqb : m);
-      out_idx[pos] = idx;
-      if constexpr (VBF16) {
-        const __nv_bfloat16 h = __float2bfloat16_rn(a);
-        reinterpret_cast<__nv_bfloat16*>(out_val)[pos] = h;
-        r[idx] = a - __bfloat162float(h);          // exact (Sterbenz), reading #8
-      } else {
-        reinterpret_cast<float*>(out_val)[pos] = a;
-        r[idx] = 0.0f;
+  const uint32_t lt = (1u << gl) - 1;
+  for (uint64_t tw = tfirst - (lane >> glog); tw < num_tiles; tw += wstride) {   // warp-uniform
+    const uint64_t t = tw + (lane >> glog);
+    const bool tv = t < num_tiles;
+    const uint2 ti = tv ? segment(t) : make_uint2(0u, 0u);
+    const uint64_t tp = tv ? tcnt[t] + __ldcg(boff + G + (t >> ts_log)) : 0;
+    uint64_t gtb = tp >> 32, eqb = tp & 0xFFFFFFFFull;
+    const uint32_t len_max = __reduce_max_sync(0xFFFFFFFFu, ti.y);
+    for (uint32_t j0 = 0; j0 < len_max; j0 += g) {
+      const uint32_t j = j0 + gl;
+      const bool in = j < ti.y;
+      float a = 0.f;
+      uint32_t idx = 0;
+      if (in) {
+        a = vsrc[(uint64_t)ti.x + j];
+        idx = mode ? ti.x + j : cand_idx[(uint64_t)ti.x + j];
       }
-    }
-  };
-  const uint64_t stride = (uint64_t)G * kThreads;
-  for (uint64_t i0 = (uint64_t)b * kThreads + threadIdx.x; i0 < N; i0 += 2 * stride) {
-    // two candidates per round, their independent loads issued together
-    const uint64_t i1 = i0 + stride;
-    const bool has1 = i1 < N;
-    const float a0v = cand_val[i0], a1v = has1 ? cand_val[i1] : 0.f;
-    const uint32_t k0 = mag_key(a0v), k1 = has1 ? mag_key(a1v) : 0u;
-    const bool s0 = k0 >= K, s1 = has1 && k1 >= K;
-    uint32_t x0 = 0, x1 = 0;
-    uint64_t S0 = 0, S1 = 0;
-    if (s0) { x0 = cand_idx[i0]; S0 = S(i0); }
-    if (s1) { x1 = cand_idx[i1]; S1 = S(i1); }
-    const uint64_t adj0 = s0 ? tloc[x0 / kTile] : 0, adj1 = s1 ? tloc[x1 / kTile] : 0;
-    if (s0) emit(i0, a0v, k0, x0, S0, adj0);
-    if (s1) emit(i1, a1v, k1, x1, S1, adj1);
-  }
-}
-
-// ---- K1d: ordered emission of the k pairs + residual fix-up on S ---------------------------
-// One CTA covers kTilesPerEmit = 256 streaming tiles. Candidate mode: one thread per tile walks its
-// (few) candidates; full mode (fallback): one warp per tile, 32 elements at a time. The per-tile
-// (count > K*, count == K*) pairs are scanned in the block and across blocks (decoupled look-back),
-// giving every selected element its output position gt_before + min(m, eq_before).
-template <bool VBF16>
-__device__ __forceinline__ void emit_one(uint64_t pos, uint32_t idx, float a, uint32_t* out_idx,
-                                         uint8_t* out_val, float* r) {
-  out_idx[pos] = idx;
-  if constexpr (VBF16) {
-    const __nv_bfloat16 h = __float2bfloat16_rn(a);
-    reinterpret_cast<__nv_bfloat16*>(out_val)[pos] = h;
-    r[idx] = a - __bfloat162float(h);              // exact (Sterbenz), reading #8
-  } else {
-    reinterpret_cast<float*>(out_val)[pos] = a;
-    r[idx] = 0.0f;
-  }
-}
-
-template <bool VBF16>
-__global__ void __launch_bounds__(kThreads) emit_kernel(float* __restrict__ r, uint64_t n, uint64_t k,
-                                                        uint32_t num_tiles, uint32_t num_emit,
-                                                        Ctl* ctl, const uint2* __restrict__ tile_info,
-                                                        const uint32_t* __restrict__ cand_idx,
-                                                        const float* __restrict__ cand_val,
-                                                        uint64_t* status, uint8_t* pairs) {
-  __shared__ uint32_t s_cnt[kTilesPerEmit][2];
-  __shared__ uint64_t s_scan[kThreads / 32];
-  __shared__ uint64_t s_bpre;
-  __shared__ uint32_t s_ticket;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const uint32_t mode = ctl->mode, K = ctl->kstar;
-  if (mode == 0) return;                           // candidate mode: emitted by select_kernel
-  const uint64_t m = ctl->m;
-  uint32_t* out_idx = reinterpret_cast<uint32_t*>(pairs);
-  uint8_t* out_val = pairs + pad16(4 * k);
-  const uint32_t lt = (1u << lane) - 1u;
-  while (true) {
-    if (tid == 0) s_ticket = atomicAdd(&ctl->emit_ticket, 1u);
-    __syncthreads();
-    const uint32_t eb = s_ticket;
-    if (eb >= num_emit) break;
-    if (eb == 0 && tid < 16) {               // zero the 16-byte padding of both sections
-      const uint64_t ip = 4 * k, ie = pad16(4 * k);
-      if (ip + tid < ie) pairs[ip + tid] = 0;
-      const uint64_t vp = pad16(4 * k) + (VBF16 ? 2 : 4) * k, ve = pad16(4 * k) + pad16((VBF16 ? 2 : 4) * k);
-      if (vp + tid < ve) pairs[vp + tid] = 0;
-    }
-    const uint32_t t_mine = eb * kTilesPerEmit + tid;
-    // phase 1: per-tile counts of keys > K* and == K*
-    uint32_t gt = 0, eq = 0;
-    if (mode == 0) {
-      if (t_mine < num_tiles) {
-        const uint2 ti = tile_info[t_mine];
-        for (uint32_t i = ti.x; i < ti.x + ti.y; ++i) {
-          const uint32_t key = mag_key(cand_val[i]);
-          gt += key > K; eq += key == K;
+      const uint32_t key = mag_key(a);
+      const bool isg = in && key > K, ise = in && key == K;
+      const uint32_t bg = (__ballot_sync(0xFFFFFFFFu, isg) >> gshift) & gmask;
+      const uint32_t be = (__ballot_sync(0xFFFFFFFFu, ise) >> gshift) & gmask;
+      const uint64_t myeq = eqb + __popc(be & lt);
+      if (isg || (ise && myeq < m)) {
+        const uint64_t pos = gtb + __popc(bg & lt) + (myeq < m ? myeq : m);
+        out_idx[pos] = idx;
+        if constexpr (VBF16) {
+          const __nv_bfloat16 h = __float2bfloat16_rn(a);
+          reinterpret_cast<__nv_bfloat16*>(out_val)[pos] = h;
+          r[idx] = a - __bfloat162float(h);        // exact (Sterbenz), reading #8
+        } else {
+          reinterpret_cast<float*>(out_val)[pos] = a;
+          r[idx] = 0.0f;
         }
       }
-    } else {
-      for (int q = 0; q < 32; ++q) {
-        const uint32_t t = eb * kTilesPerEmit + warp * 32 + q;
-        uint32_t g2 = 0, e2 = 0;
-        if (t < num_tiles) {
-          const uint64_t s = (uint64_t)t * kTile, e = s + kTile < n ? s + kTile : n;
-          for (uint64_t i = s + lane; i < e; i += 32) {
-            const uint32_t key = mag_key(r[i]);
-            g2 += key > K; e2 += key == K;
-          }
-        }
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-          g2 += __shfl_xor_sync(0xFFFFFFFFu, g2, o);
-          e2 += __shfl_xor_sync(0xFFFFFFFFu, e2, o);
-        }
-        if (lane == q) { gt = g2; eq = e2; }
-      }
+      gtb += __popc(bg);
+      eqb += __popc(be);
     }
-    uint64_t tot;
-    const uint64_t pre = block_exclusive_scan(((uint64_t)gt << 31) | eq, s_scan, &tot);
-    if (warp == 0) {
-      const uint64_t bpre = lookback_exclusive(status, eb, tot);
-      if (lane == 0) s_bpre = bpre;
-    }
-    __syncthreads();
-    const uint64_t mypre = s_bpre + pre;
-    // phase 2: emit in index order
-    if (mode == 0) {
-      if (t_mine < num_tiles) {
-        uint64_t gtb = mypre >> 31, eqb = mypre & 0x7FFFFFFFull;
-        const uint2 ti = tile_info[t_mine];
-        for (uint32_t i = ti.x; i < ti.x + ti.y; ++i) {
-          const float a = cand_val[i];
-          const uint32_t key = mag_key(a);
-          if (key > K) {
-            emit_one<VBF16>(gtb + (eqb < m ? eqb : m), cand_idx[i], a, out_idx, out_val, r);
-            ++gtb;
-          } else if (key == K) {
-            if (eqb < m) emit_one<VBF16>(gtb + eqb, cand_idx[i], a, out_idx, out_val, r);
-            ++eqb;
-          }
-        }
-      }
-    } else {
-      s_cnt[tid][0] = (uint32_t)(mypre >> 31);
-      s_cnt[tid][1] = (uint32_t)(mypre & 0x7FFFFFFFull);
-      __syncthreads();
-      for (int q = 0; q < 32; ++q) {
-        const uint32_t t = eb * kTilesPerEmit + warp * 32 + q;
-        if (t >= num_tiles) break;
-        uint64_t gtb = s_cnt[warp * 32 + q][0], eqb = s_cnt[warp * 32 + q][1];
-        const uint64_t s = (uint64_t)t * kTile, e = s + kTile < n ? s + kTile : n;
-        for (uint64_t i0 = s; i0 < e; i0 += 32) {
-          const uint64_t i = i0 + lane;
-          const bool valid = i < e;
-          const float a = valid ? r[i] : 0.f;
-          const uint32_t key = mag_key(a);
-          const bool isgt = valid && key > K, iseq = valid && key == K;
-          const uint32_t bg = __ballot_sync(0xFFFFFFFFu, isgt), be = __ballot_sync(0xFFFFFFFFu, iseq);
-          const uint64_t gb = gtb + __popc(bg & lt), eqbefore = eqb + __popc(be & lt);
-          if (isgt || (iseq && eqbefore < m))
-            emit_one<VBF16>(gb + (eqbefore < m ? eqbefore : m), (uint32_t)i, a, out_idx, out_val, r);
-          gtb += __popc(bg);
-          eqb += __popc(be);
-        }
-      }
-    }
-    __syncthreads();
   }
 }
 
@@ -707,7 +595,6 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
     float* rr = residual;
     uint32_t *h0 = reinterpret_cast<uint32_t*>(w + L.h0), *h1 = reinterpret_cast<uint32_t*>(w + L.h1),
              *h2 = reinterpret_cast<uint32_t*>(w + L.h2);
-    uint64_t* sloc = reinterpret_cast<uint64_t*>(w + L.sloc);
     uint64_t* tloc = reinterpret_cast<uint64_t*>(w + L.tloc);
     uint64_t* boff = reinterpret_cast<uint64_t*>(w + L.boff);
     uint8_t* pp = static_cast<uint8_t*>(pairs);
@@ -716,21 +603,13 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
     uint32_t cap = L.cap, nt = L.num_tiles;
     void* args[] = {(void*)&rr, (void*)&n, (void*)&k, (void*)&ctl, (void*)&cval, (void*)&cidx_c,
                     (void*)&tiles_c, (void*)&nt, (void*)&cap, (void*)&h0, (void*)&h1, (void*)&h2,
-                    (void*)&sloc, (void*)&tloc, (void*)&boff, (void*)&pp};
+                    (void*)&tloc, (void*)&boff, (void*)&pp};
     ProfScope prof("compress_select", s);
     const void* fn = vdt == LOWDIFF_BF16 ? (const void*)select_kernel<true> : (const void*)select_kernel<false>;
     LD_CUDA(cudaLaunchCooperativeKernel(fn, sel_grid, kThreads, args, 0, s), "select launch");
     note_launch();
   }
 
-  int egrid = (int)(L.num_emit < 4u * kNumSMs ? L.num_emit : 4u * kNumSMs);
-  uint64_t* status = reinterpret_cast<uint64_t*>(w + L.status);
-  if (vdt == LOWDIFF_BF16)
-    LD_LAUNCH("compress_emit", s, emit_kernel<true>, egrid, kThreads, 0, residual, n, k, L.num_tiles,
-              L.num_emit, ctl, tiles, cidx, cval, status, static_cast<uint8_t*>(pairs));
-  else
-    LD_LAUNCH("compress_emit", s, emit_kernel<false>, egrid, kThreads, 0, residual, n, k, L.num_tiles,
-              L.num_emit, ctl, tiles, cidx, cval, status, static_cast<uint8_t*>(pairs));
   return cuda_status(cudaGetLastError(), "compress launch");
 }
 

@@ -1,7 +1,7 @@
 #!/bin/bash
 # Bench every BASELINE config at N=1 (GPU box). Usage: bench_all.sh <tag>
 TAG=${1:-r01}; OUT=gpurun_out; mkdir -p $OUT
-for C in 1 2 3 4 5; do
+for C in ${CONFIGS:-1 2 3 4 5}; do
   EXTRA=""
   [ $C = 5 ] && EXTRA="--grad-pool 4"
   [ $C = 4 ] && EXTRA="--grad-pool 8"
