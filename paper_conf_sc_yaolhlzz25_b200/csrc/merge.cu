@@ -151,8 +151,7 @@ struct DenseSmem {
   uint32_t cnt[kW];              // entries per slot
 };
 struct SparseSmem {
-  uint64_t sk[kCap];             // (idx - w0) << 40 | list << 32 | load position; sorted in place
-  float val[kCap];               // values at their load position
+  uint64_t sk[2][kCap];          // (idx - w0) << 40 | list << 32 | load position; merge ping-pong
 };
 union ItemSmem {
   DenseSmem d;
@@ -205,50 +204,60 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
     const uint32_t e0 = s_e0;
     uint64_t tot;
     if (E <= (uint32_t)kCap) {
-      // ---- sparse item: load, then a shared-memory bitonic sort on the unique composite
-      //      (index, list) key — equal indices end up in list (rank / iteration) order ----
-      uint32_t Np = 32;
-      while (Np < E) Np <<= 1;
-      for (uint32_t x = tid; x < Np; x += kThreads) {
-        if (x < E) {
-          int a = 0, b = L - 1;                    // list l with s_off[l] <= x < s_off[l+1]
-          while (a < b) {
-            const int mid = (a + b + 1) >> 1;
-            if (s_off[mid] <= x) a = mid; else b = mid - 1;
-          }
-          const uint64_t e = s_beg[a] + (x - s_off[a]);
-          const uint32_t key = ls.list[a].idx[e] - (uint32_t)w0;
-          sm.s.sk[x] = ((uint64_t)key << 40) | ((uint64_t)a << 32) | x;
-          sm.s.val[x] = list_val<BF16>(ls, a, e);
-        } else {
-          sm.s.sk[x] = ~0ull;                      // padding sorts last
+      // ---- sparse item: load the lists' segments (each sorted by index) as runs of unique
+      //      composite keys (index, list), then merge runs pairwise, ceil(log2 L) rounds: a key's
+      //      rank in the merged run = its rank in its own run + the number of smaller keys in the
+      //      partner run (binary search). Equal indices end up in list (rank / iteration) order.
+      for (uint32_t x = tid; x < E; x += kThreads) {
+        int a = 0, b = L - 1;                      // list l with s_off[l] <= x < s_off[l+1]
+        while (a < b) {
+          const int mid = (a + b + 1) >> 1;
+          if (s_off[mid] <= x) a = mid; else b = mid - 1;
         }
+        const uint64_t e = s_beg[a] + (x - s_off[a]);
+        const uint32_t key = ls.list[a].idx[e] - (uint32_t)w0;
+        sm.s.sk[0][x] = ((uint64_t)key << 40) | ((uint64_t)a << 32) | x;
       }
       __syncthreads();
-      for (uint32_t kk = 2; kk <= Np; kk <<= 1) {
-        for (uint32_t j = kk >> 1; j > 0; j >>= 1) {
-          for (uint32_t i = tid; i < Np / 2; i += kThreads) {
-            const uint32_t lo_ = 2 * j * (i / j) + (i % j), hi_ = lo_ + j;
-            const uint64_t A = sm.s.sk[lo_], Bv = sm.s.sk[hi_];
-            if ((A > Bv) == ((lo_ & kk) == 0)) { sm.s.sk[lo_] = Bv; sm.s.sk[hi_] = A; }
+      int cur = 0;
+      for (int w = 1; w < L; w <<= 1, cur ^= 1) {  // runs of w lists -> runs of 2w lists
+        const uint64_t* A = sm.s.sk[cur];
+        uint64_t* Bo = sm.s.sk[cur ^ 1];
+        for (uint32_t x = tid; x < E; x += kThreads) {
+          const uint64_t key = A[x];
+          const int q = (int)((key >> 32) & 0xFFu) / w;   // own run
+          const int pq = q ^ 1;                            // partner run
+          const uint32_t own_s = s_off[q * w];
+          const uint32_t ps = s_off[pq * w < L ? pq * w : L];
+          const uint32_t pe = s_off[(pq + 1) * w < L ? (pq + 1) * w : L];
+          uint32_t pos = ps, len = pe - ps;               // lower_bound of key in A[ps, pe)
+          while (len > 0) {
+            const uint32_t half = len >> 1;
+            if (A[pos + half] < key) { pos += half + 1; len -= half + 1; } else { len = half; }
           }
-          __syncthreads();
+          Bo[s_off[(q & ~1) * w] + (x - own_s) + (pos - ps)] = key;
         }
+        __syncthreads();
       }
+      const uint64_t* S = sm.s.sk[cur];
+      auto val_of = [&](uint64_t skr) -> float {  // the value of a key, from its list (L2-warm)
+        const int l = (int)((skr >> 32) & 0xFFu);
+        return list_val<BF16>(ls, l, s_beg[l] + ((uint32_t)skr - s_off[l]));
+      };
       uint32_t my_u = 0;
 #pragma unroll
       for (int j = 0; j < kPosPerThread; ++j) {
         const uint32_t r = tid * kPosPerThread + j;
-        if (r < E && (r == 0 || (sm.s.sk[r - 1] >> 40) != (sm.s.sk[r] >> 40))) ++my_u;
+        if (r < E && (r == 0 || (S[r - 1] >> 40) != (S[r] >> 40))) ++my_u;
       }
       uint32_t u = e0 + (uint32_t)block_exclusive_scan(my_u, s_scan, &tot);
 #pragma unroll
       for (int j = 0; j < kPosPerThread; ++j) {
         const uint32_t r = tid * kPosPerThread + j;
         if (r >= E) break;
-        const uint64_t skr = sm.s.sk[r];
+        const uint64_t skr = S[r];
         const uint32_t key = (uint32_t)(skr >> 40);
-        const bool head = r == 0 || (sm.s.sk[r - 1] >> 40) != key;
+        const bool head = r == 0 || (S[r - 1] >> 40) != key;
         if (KIND == kMergeStack) {
           if (head) {
             stg_idx[u] = (uint32_t)(w0 + key);
@@ -256,11 +265,11 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
             ++u;
           }
           out_it[e0 + r] = (uint8_t)(skr >> 32);
-          out_ent[e0 + r] = sm.s.val[(uint32_t)skr];
+          out_ent[e0 + r] = val_of(skr);
         } else if (head) {
-          float sum = sm.s.val[(uint32_t)skr];     // fold the run in list order
-          for (uint32_t r2 = r + 1; r2 < E && (sm.s.sk[r2] >> 40) == key; ++r2)
-            sum = sum + sm.s.val[(uint32_t)sm.s.sk[r2]];
+          float sum = val_of(skr);                 // fold the run in list order
+          for (uint32_t r2 = r + 1; r2 < E && (S[r2] >> 40) == key; ++r2)
+            sum = sum + val_of(S[r2]);
           stg_idx[u] = (uint32_t)(w0 + key);
           stg_val[u] = __float_as_uint(sum);
           ++u;
