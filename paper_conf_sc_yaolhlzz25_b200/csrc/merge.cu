@@ -89,8 +89,8 @@ __device__ __forceinline__ float list_val(const ListSet& ls, int l, uint64_t e) 
 // ---- K2p: work-item plan (one CTA) -----------------------------------------------------------------
 // items[i] = (first fine window, number of fine windows).
 __global__ void __launch_bounds__(kPlanThreads) plan_kernel(int L, const uint32_t* __restrict__ starts,
-                                                            uint32_t num_w, uint32_t G, MCtl* ctl,
-                                                            uint2* __restrict__ items) {
+                                                            uint32_t num_w, uint32_t G, uint32_t sparse_max,
+                                                            MCtl* ctl, uint2* __restrict__ items) {
   __shared__ uint32_t s_warp[kPlanThreads / 32];
   __shared__ uint32_t s_carry;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -119,7 +119,7 @@ __global__ void __launch_bounds__(kPlanThreads) plan_kernel(int L, const uint32_
         const uint32_t* st = starts + (uint64_t)l * (num_w + 1);
         e += st[fe] - st[fs];
       }
-      cnt = (e <= (uint64_t)kCap || fe - fs == 1) ? 1u : fe - fs;
+      cnt = (e <= (uint64_t)sparse_max || fe - fs == 1) ? 1u : fe - fs;
     }
     uint32_t incl = cnt;
 #pragma unroll
@@ -166,7 +166,7 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
                                                          uint32_t* __restrict__ stg_idx,
                                                          uint32_t* __restrict__ stg_val,
                                                          uint8_t* __restrict__ out_it,
-                                                         float* __restrict__ out_ent) {
+                                                         float* __restrict__ out_ent, uint32_t sparse_max) {
   __shared__ ItemSmem sm;
   __shared__ uint32_t s_beg[kMaxLists], s_len[kMaxLists], s_off[kMaxLists + 1];
   __shared__ uint64_t s_scan[kThreads / 32];
@@ -203,7 +203,7 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
     const uint32_t E = (uint32_t)tot_e;
     const uint32_t e0 = s_e0;
     uint64_t tot;
-    if (E <= (uint32_t)kCap) {
+    if (E <= sparse_max) {
       // ---- sparse item: load the lists' segments (each sorted by index) as runs of unique
       //      composite keys (index, list), then merge runs pairwise, ceil(log2 L) rounds: a key's
       //      rank in the merged run = its rank in its own run + the number of smaller keys in the
@@ -617,7 +617,11 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
   const double per_w = (double)max_entries / (double)M.num_w;
   uint32_t G = 1;
   while (G < 4096 && (double)(2 * G) * per_w <= kCap / 2) G <<= 1;     // key < 2^24
-  LD_LAUNCH("merge_plan", s, plan_kernel, 1, kPlanThreads, 0, ls.L, starts, M.num_w, G, ctl, items);
+  uint32_t sparse_max = kCap;       // items with more entries take the dense (one window) path
+  if (const char* e = getenv("LOWDIFF_MERGE_SPARSE_MAX")) sparse_max = (uint32_t)atoi(e);
+  if (sparse_max > (uint32_t)kCap) sparse_max = kCap;
+  LD_LAUNCH("merge_plan", s, plan_kernel, 1, kPlanThreads, 0, ls.L, starts, M.num_w, G, sparse_max, ctl,
+            items);
 
   const int grid = (int)(M.num_w < 6u * kNumSMs ? M.num_w : 6u * kNumSMs);   // 6 CTAs/SM (37 KB smem)
   uint32_t* ucnt = reinterpret_cast<uint32_t*>(w + M.ucnt);
@@ -630,16 +634,16 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
   const char* cls = record ? "merge" : "coalesce";
   if (kind == kCoalesce && ls.bf16)
     LD_LAUNCH(cls, s, (merge_kernel<kCoalesce, true>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
-              ucnt, epre, sidx, sval, oit, oent);
+              ucnt, epre, sidx, sval, oit, oent, sparse_max);
   else if (kind == kCoalesce)
     LD_LAUNCH(cls, s, (merge_kernel<kCoalesce, false>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
-              ucnt, epre, sidx, sval, oit, oent);
+              ucnt, epre, sidx, sval, oit, oent, sparse_max);
   else if (kind == kMergeSum)
     LD_LAUNCH(cls, s, (merge_kernel<kMergeSum, false>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
-              ucnt, epre, sidx, sval, oit, oent);
+              ucnt, epre, sidx, sval, oit, oent, sparse_max);
   else
     LD_LAUNCH(cls, s, (merge_kernel<kMergeStack, false>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
-              ucnt, epre, sidx, sval, oit, oent);
+              ucnt, epre, sidx, sval, oit, oent, sparse_max);
   LD_LAUNCH(cls, s, ucount_scan_kernel, 1, kPlanThreads, 0, ls, M.num_w, starts, ctl, ucnt, upre,
             kind == kCoalesce ? d_out_nnz : nullptr);
   uint32_t* didx = record ? reinterpret_cast<uint32_t*>(w + M.widx) : out_idx;
