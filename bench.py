@@ -348,6 +348,26 @@ def run_ours(args, cfg):
                 "alg_bytes_per_launch": alg_bytes, "launch_ms": cs_ms / cs_n if cs_n else None,
                 "peak_source": peak_note}
 
+    # ---- the replay kernel against its own bound (HBM bytes and, for Adam, the MUFU floor) ----
+    replay_roof = None
+    rp_ms, rp_n = prof.get("replay_dense", (0.0, 0))
+    if rp_n:
+        nloc = hi - lo
+        sb = {"sgd": 8, "momentum": 16, "adam": 24}[cfg.opt]          # read + write of x (m, v)
+        alg = sb * nloc + int(rec_bytes)                                 # + the chain's records
+        t_s = rp_ms / args.steps * 1e-3                                  # per step (one chain)
+        replay_roof = {"kernel": "replay_dense", "alg_bytes_per_step": alg,
+                       "achieved_gbs": alg / t_s / 1e9, "hbm_frac": alg / t_s / 1e9 / hbm_peak,
+                       "ms_per_step": rp_ms / args.steps}
+        if cfg.opt == "adam":
+            # 2 MUFU ops (rsqrt, rcp) per parameter-step at 16/clk/SM on 148 SMs
+            f_mhz = (clk or {}).get("sm_mhz") or 1965.0
+            floor_s = 2.0 * nloc * R * B / (148 * 16 * f_mhz * 1e6)
+            replay_roof.update({"bound": "alu", "alu_floor_ms": floor_s * 1e3, "alu_frac": floor_s / t_s,
+                                "alu_peak": f"MUFU 16/clk/SM x 148 SMs at {f_mhz:.0f} MHz"})
+        else:
+            replay_roof["bound"] = "alu" if replay_roof["hbm_frac"] < 0.5 else "hbm"
+
     # ---- e2e: same metric through the public API with host buffers (pinned H2D of every gradient) ----
     e2e = None
     if not args.no_e2e:
@@ -395,7 +415,7 @@ def run_ours(args, cfg):
                 "timing": {"build_phase": "one CUDA graph per step" if graph is not None else "eager launches",
                            "profiled_ms_per_step": pms / args.steps,
                            "profiled": "separate pass, eager launches, CUDA events around every kernel"},
-                "roofline": roofline, "kernels": kernels, "cpu_baseline": cpu, "e2e": e2e,
+                "roofline": roofline, "replay_roofline": replay_roof, "kernels": kernels, "cpu_baseline": cpu, "e2e": e2e,
                 "gpu_launches": int(launches), "clocks": clk}
         print(json.dumps(line), flush=True)
     if comm is not None:

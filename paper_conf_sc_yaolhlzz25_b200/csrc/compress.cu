@@ -591,7 +591,11 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
     if (const char* e = getenv("LOWDIFF_SELECT_PER_SM")) want = atoi(e);
     if (want < 1) want = 1;
     if (want > sel_max) want = sel_max;
-    const int sel_grid = want * kNumSMs;
+    int sel_grid = want * kNumSMs;
+    if (const char* e = getenv("LOWDIFF_SELECT_GRID")) {   // experiments: explicit CTA count
+      const int gq = atoi(e);
+      if (gq >= 1 && gq <= sel_max * kNumSMs && gq <= kMaxSelectBlocks) sel_grid = gq;
+    }
     float* rr = residual;
     uint32_t *h0 = reinterpret_cast<uint32_t*>(w + L.h0), *h1 = reinterpret_cast<uint32_t*>(w + L.h1),
              *h2 = reinterpret_cast<uint32_t*>(w + L.h2);
