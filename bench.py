@@ -222,16 +222,36 @@ def run_ours(args, cfg):
     copy_stream = torch.cuda.Stream()
     t_iter = [0]
 
+    h2d_stream = torch.cuda.Stream()
+    ev_copy = [torch.cuda.Event() for _ in range(2)]
+    ev_free = [torch.cuda.Event() for _ in range(2)]
+
     def build_phase(h2d=None):
-        """B iterations of compress -> sparse all-gather + coalesce of this rank's shard -> ring."""
+        """B iterations of compress -> sparse all-gather + coalesce of this rank's shard -> ring.
+        e2e (h2d given): iteration j's gradient is copied from pinned host memory on a copy stream
+        into one of two device buffers, overlapping the compute of iteration j-1."""
+        cs = torch.cuda.current_stream()              # the graph-capture stream when captured
         for j in range(B):
-            if h2d is not None:               # e2e: this iteration's gradient from pinned host memory
-                h2d[0][j % len(h2d[0])].copy_(h2d[1][j % len(h2d[1])], non_blocking=True)
-                g = h2d[0][j % len(h2d[0])]
+            if h2d is not None:
+                D = len(h2d[0])
+                d = j % D
+                if j == 0:
+                    h2d_stream.wait_stream(cs)        # buffers free: the previous batch is done
+                elif j >= D:
+                    h2d_stream.wait_event(ev_free[d])
+                with torch.cuda.stream(h2d_stream):
+                    h2d[0][d].copy_(h2d[1][j % len(h2d[1])], non_blocking=True)
+                ev_copy[d].record(h2d_stream)
+                cs.wait_event(ev_copy[d])
+                g = h2d[0][d]
             else:
                 g = grads[j % len(grads)]
             ld.compress(g, r, k, vdt=cfg.vdt, pairs=pairs)
+            if h2d is not None:
+                ev_free[d].record(cs)
             ld.allgather_sparse(comm, pairs, k, cfg.vdt, lo, hi, True, *ring[j])
+        if h2d is not None:
+            cs.wait_stream(h2d_stream)
 
     def checkpoint_phase(b):
         """Batch merge -> record b -> async D2H stage (copy stream); returns the record's bytes."""
