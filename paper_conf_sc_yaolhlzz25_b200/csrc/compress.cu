@@ -4,7 +4,7 @@
 // Design: the only HBM-heavy step is one fused streaming pass
 //   a = g + r;  r <- a;  if |a| >= T_est: append (i, a) to a candidate buffer
 // which moves the algorithmic floor of 12n bytes (fp32 g) / 10n (bf16 g). T_est comes from a
-// small stratified sample of |g + r| (8-element micro-chunks, >= 1024 n/k of them) so the
+// small stratified sample of |g + r| (8-element micro-chunks, >= 512 n/k keys) so the
 // candidates number ~1.3-2 k. One cooperative kernel then does the rest: an exact 3-digit radix
 // select (12/10/9 bits of the 31-bit key) over the candidates finds the k-th key K* and the number
 // m of K*-ties to keep, and an ordered emission (per-tile counts, a scan over tiles, ballot
@@ -166,7 +166,7 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(const void* g, const f
   __threadfence();
   // Need: exhaustive -> exactly k (threshold = the bin's lower edge: exact, >= k candidates);
   // sampled -> 1.3 x the expected sample count above the k-th key (+8): the candidates land at
-  // ~1.3 k, >8 sigma above k for S >= 2048 n / k. Within the 12.5 %-wide bin the threshold is
+  // ~1.3 k, >7 sigma above k for S >= 512 n / k. Within the 12.5 %-wide bin the threshold is
   // placed by an exponential-density model fitted to this bin and the next one up (the tail
   // density falls steeply, so a uniform model lands too high), then moved 10 % toward the lower
   // edge as a safety margin.
@@ -542,10 +542,10 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   Ctl* ctl = reinterpret_cast<Ctl*>(w + L.ctl);
   LD_CUDA(cudaMemsetAsync(w, 0, L.zero_end, s), "memset compress workspace");
 
-  // sample size: >= 1024 expected keys above the k-th (S >= 1024 n / k: the 1.3x target is then
-  // ~9 sigma above k), >= 64 Ki, power of 2
+  // sample size: >= 512 expected keys above the k-th (S >= 512 n / k: the 1.3x target, ~666
+  // sampled keys, is then ~7.5 sigma of the count above k), >= 64 Ki, power of 2
   uint64_t S = 65536;
-  while ((double)S * (double)k < 1024.0 * (double)n && S < (1ull << 26)) S <<= 1;
+  while ((double)S * (double)k < 512.0 * (double)n && S < (1ull << 26)) S <<= 1;
   const int exhaustive = (S >= n / 2) ? 1 : 0;
   const uint32_t micro = exhaustive ? (uint32_t)((n + 7) / 8) : (uint32_t)(S / 8);
   const double stride = exhaustive ? 1.0 : (double)(n / 8) / (double)micro;
