@@ -294,6 +294,168 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
   }
 }
 
+// ---- K1b': the streaming pass with 1-D TMA bulk copies -------------------------------------
+// Same per-tile work as stream_kernel, but the g and r tiles of this CTA's next kStages tiles are
+// in flight as cp.async.bulk copies (one elected thread, completion on an mbarrier per stage)
+// while the current tile is scanned, so the loads never wait behind the block scan's barriers.
+// Full tiles only; the ragged last tile (if any) takes the direct-load path.
+#ifndef LOWDIFF_STREAM_STAGES
+#define LOWDIFF_STREAM_STAGES 2
+#endif
+constexpr int kStages = LOWDIFF_STREAM_STAGES;
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "LAB_WAIT:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra LAB_WAIT;\n}" :: "r"(bar), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               :: "r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+
+template <bool BF16>
+__global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __restrict__ g,
+                                                              float* __restrict__ r, uint64_t n,
+                                                              uint32_t num_tiles, Ctl* ctl,
+                                                              uint2* __restrict__ tile_info,
+                                                              uint32_t* __restrict__ cand_idx,
+                                                              float* __restrict__ cand_val, uint32_t cap) {
+  constexpr uint32_t kGB = kTile * (BF16 ? 2 : 4), kRB = kTile * 4, kSB = kGB + kRB;
+  extern __shared__ __align__(128) uint8_t s_tiles[];          // kStages x {g tile, r tile}
+  __shared__ __align__(8) uint64_t s_bar[kStages];
+  __shared__ uint64_t s_scan[2][kThreads / 32];
+  __shared__ uint32_t s_base[2];
+  const uint32_t T = ctl->t_est;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t full_tiles = (uint32_t)(n / kTile);
+  auto issue = [&](uint32_t it) {                              // this CTA's it-th tile -> its stage
+    const uint32_t tile = blockIdx.x + it * gridDim.x;
+    if (tile >= full_tiles) return;
+    const uint32_t st = it % kStages, bar = smem_u32(&s_bar[st]);
+    const uint32_t dst = smem_u32(s_tiles + st * kSB);
+    mbar_expect_tx(bar, kSB);
+    bulk_g2s(dst, static_cast<const uint8_t*>(g) + (uint64_t)tile * kGB, kGB, bar);
+    bulk_g2s(dst + kGB, reinterpret_cast<const uint8_t*>(r) + (uint64_t)tile * kRB, kRB, bar);
+  };
+  if (tid == 0) {
+    for (int s = 0; s < kStages; ++s) mbar_init(smem_u32(&s_bar[s]), 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    for (uint32_t it = 0; it < (uint32_t)kStages; ++it) issue(it);
+  }
+  __syncthreads();
+  int par = 0;
+  uint32_t it = 0;
+  for (uint32_t tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, par ^= 1, ++it) {
+    const uint64_t base = (uint64_t)tile * kTile;
+    float a[4][4];
+    uint32_t flags = 0;
+    if (tile < full_tiles) {
+      const uint32_t st = it % kStages;
+      mbar_wait(smem_u32(&s_bar[st]), (it / kStages) & 1u);
+      const uint8_t* sg = s_tiles + st * kSB;
+      const float* sr = reinterpret_cast<const float*>(sg + kGB);
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        const int o = c * 1024 + tid * 4;
+        float4 gv;
+        if constexpr (BF16) {
+          const uint2 u = *reinterpret_cast<const uint2*>(sg + 2 * o);
+          gv = make_float4(__uint_as_float(u.x << 16), __uint_as_float(u.x & 0xFFFF0000u),
+                           __uint_as_float(u.y << 16), __uint_as_float(u.y & 0xFFFF0000u));
+        } else {
+          gv = *reinterpret_cast<const float4*>(sg + 4 * o);
+        }
+        const float4 rv = *reinterpret_cast<const float4*>(sr + o);
+        a[c][0] = gv.x + rv.x; a[c][1] = gv.y + rv.y; a[c][2] = gv.z + rv.z; a[c][3] = gv.w + rv.w;
+      }
+    } else {
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const uint64_t i = base + c * 1024 + tid * 4 + e;
+          a[c][e] = i < n ? load_g1<BF16>(g, i) + r[i] : 0.f;
+        }
+    }
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+      const uint64_t i = base + c * 1024 + tid * 4;
+      if (tile < full_tiles) {
+        __stcs(reinterpret_cast<float4*>(r + i), make_float4(a[c][0], a[c][1], a[c][2], a[c][3]));
+#pragma unroll
+        for (int e = 0; e < 4; ++e) flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
+      } else {
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          if (i + e < n) {
+            r[i + e] = a[c][e];
+            flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
+          }
+      }
+    }
+    // Order-preserving compaction: one block scan of 4 x 16-bit per-vector counts.
+    uint64_t packed = 0;
+#pragma unroll
+    for (int c = 0; c < 4; ++c) packed |= (uint64_t)__popc((flags >> (4 * c)) & 0xFu) << (16 * c);
+    uint64_t incl = packed;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      uint64_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+      if (lane >= o) incl += y;
+    }
+    if (lane == 31) s_scan[par][warp] = incl;
+    __syncthreads();                                  // every thread is done reading this stage
+    if (tid == 0) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      issue(it + kStages);                            // refill the stage just consumed
+    }
+    uint64_t warp_off = 0, tot = 0;
+#pragma unroll
+    for (int w = 0; w < kThreads / 32; ++w) {
+      uint64_t t = s_scan[par][w];
+      warp_off += (w < warp) ? t : 0;
+      tot += t;
+    }
+    const uint64_t excl = warp_off + incl - packed;
+    uint32_t vec_base[4], total = 0;
+#pragma unroll
+    for (int c = 0; c < 4; ++c) { vec_base[c] = total; total += (uint32_t)((tot >> (16 * c)) & 0xFFFF); }
+    if (tid == 0) {
+      uint32_t b = total ? atomicAdd(&ctl->cand_count, total) : 0u;
+      s_base[par] = b;
+      tile_info[tile] = make_uint2(b, total);
+    }
+    __syncthreads();
+    if (total) {
+      const uint32_t b = s_base[par];
+      if ((uint64_t)b + total <= cap && flags) {
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          uint32_t pos = b + vec_base[c] + (uint32_t)((excl >> (16 * c)) & 0xFFFF);
+#pragma unroll
+          for (int e = 0; e < 4; ++e)
+            if (flags & (1u << (c * 4 + e))) {
+              cand_idx[pos] = (uint32_t)(base + c * 1024 + tid * 4 + e);
+              cand_val[pos] = a[c][e];
+              ++pos;
+            }
+        }
+      }
+    }
+  }
+}
+
 // ---- K1c: exact radix select over the candidates (or the full array) ------------------------
 // One cooperative launch runs the three digit passes (12 + 10 + 9 bits of the 31-bit key) with a
 // grid barrier after each histogram; every CTA then redoes the tiny 'find' on the L2-resident
@@ -505,6 +667,25 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
 int g_stream_blocks_f32 = 0, g_stream_blocks_bf16 = 0;
 uint32_t g_force_t = 0xFFFFFFFFu;       // test hook: override the sampled threshold
 
+int g_tma_blocks_f32 = 0, g_tma_blocks_bf16 = 0;
+int stream_tma_smem(bool bf16) { return kStages * kTile * ((bf16 ? 2 : 4) + 4); }
+int stream_tma_blocks(bool bf16) {
+  int& cache = bf16 ? g_tma_blocks_bf16 : g_tma_blocks_f32;
+  if (!cache) {
+    const int smem = stream_tma_smem(bf16);
+    int per_sm = 0;
+    if (bf16) {
+      cudaFuncSetAttribute(stream_tma_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, stream_tma_kernel<true>, kThreads, smem);
+    } else {
+      cudaFuncSetAttribute(stream_tma_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, stream_tma_kernel<false>, kThreads, smem);
+    }
+    cache = (per_sm > 0 ? per_sm : 1) * kNumSMs;
+  }
+  return cache;
+}
+
 int stream_blocks(bool bf16) {
   int& cache = bf16 ? g_stream_blocks_bf16 : g_stream_blocks_f32;
   if (!cache) {
@@ -566,14 +747,31 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   uint32_t* cidx = reinterpret_cast<uint32_t*>(w + L.cand_idx);
   float* cval = reinterpret_cast<float*>(w + L.cand_val);
   const bool bf = gdt == LOWDIFF_BF16;
-  int grid = stream_blocks(bf);
-  if ((uint32_t)grid > L.num_tiles) grid = (int)L.num_tiles;
-  if (bf)
-    LD_LAUNCH("compress_stream", s, stream_kernel<true>, grid, kThreads, 0, grad, residual, n,
-              L.num_tiles, ctl, tiles, cidx, cval, L.cap);
-  else
-    LD_LAUNCH("compress_stream", s, stream_kernel<false>, grid, kThreads, 0, grad, residual, n,
-              L.num_tiles, ctl, tiles, cidx, cval, L.cap);
+  static int use_tma = -1;
+  if (use_tma < 0) {
+    const char* e = getenv("LOWDIFF_STREAM_TMA");
+    use_tma = e ? atoi(e) : 0;
+  }
+  if (use_tma) {
+    int grid = stream_tma_blocks(bf);
+    if ((uint32_t)grid > L.num_tiles) grid = (int)L.num_tiles;
+    const int smem = stream_tma_smem(bf);
+    if (bf)
+      LD_LAUNCH("compress_stream", s, stream_tma_kernel<true>, grid, kThreads, smem, grad, residual, n,
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap);
+    else
+      LD_LAUNCH("compress_stream", s, stream_tma_kernel<false>, grid, kThreads, smem, grad, residual, n,
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap);
+  } else {
+    int grid = stream_blocks(bf);
+    if ((uint32_t)grid > L.num_tiles) grid = (int)L.num_tiles;
+    if (bf)
+      LD_LAUNCH("compress_stream", s, stream_kernel<true>, grid, kThreads, 0, grad, residual, n,
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap);
+    else
+      LD_LAUNCH("compress_stream", s, stream_kernel<false>, grid, kThreads, 0, grad, residual, n,
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap);
+  }
 
   {
     static int sel_max = 0;                        // occupancy limit (CTAs per SM), both variants
