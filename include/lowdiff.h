@@ -222,13 +222,43 @@ lowdiff_status lowdiff_replay(lowdiff_state* st, const lowdiff_opt* opt,
                               uint64_t ws_bytes, lowdiff_stream_t stream);
 
 /* ---------------------------------------------------------------------------------------------
+ * Checkpointing configuration model (§3.5 "Optimizing Checkpointing Configuration", P:318-350;
+ * SURVEY §8(f) NEXT-3). Host-only arithmetic (fp64), no stream, no device memory.
+ *
+ * Parameters, all > 0 and finite (EINVAL otherwise), in ONE consistent time unit — the paper's
+ * model counts the wasted work of b batched iterations as b/2 time units, i.e. the unit
+ * is one training iteration (reading #29):
+ *   N   GPUs;  M  mean time between failures;  W  checkpoint write bandwidth (bytes per unit);
+ *   S   full checkpoint size (bytes);  T  total run time;  R_F  time to load a full checkpoint;
+ *   R_D time to merge (replay) one differential checkpoint onto the full one.
+ * Variables: f = full checkpoints per unit of time (FCF = 1/f iterations between them), b =
+ * batching size (differentials per batched write).
+ *
+ * lowdiff_wasted_time: Eq. 3
+ *   T_wasted(f, b) = (N T / M) (b/2 + R_F + (R_D/2) (1/(f b) - 1)) + N T S f / W
+ * lowdiff_optimal_config: Eq. 5, the stationary point of Eq. 4
+ *   f* = cbrt(R_D W^2 / (4 S^2 M^2)),  b* = cbrt(2 S R_D M / W)
+ *   and the integer configuration (fcf >= batch >= 1) minimising Eq. 3: batch is floor/ceil(b*),
+ *   fcf is floor/ceil of sqrt(2 S M batch / (R_D W)) (the b = batch root of Eq. 4's first line),
+ *   clamped to >= batch — exact because Eq. 3 is convex in fcf and its minimum over fcf is convex
+ *   in b (ties: smaller fcf, then smaller batch). Outputs are host pointers; any may be NULL.
+ * ------------------------------------------------------------------------------------------- */
+typedef struct lowdiff_config_model {
+  double N, M, W, S, T, R_F, R_D;
+} lowdiff_config_model;
+
+lowdiff_status lowdiff_wasted_time(const lowdiff_config_model* m, double f, double b, double* t_wasted);
+lowdiff_status lowdiff_optimal_config(const lowdiff_config_model* m, double* f_star, double* b_star,
+                                      uint32_t* fcf, uint32_t* batch);
+
+/* ---------------------------------------------------------------------------------------------
  * Instrumentation (bench/tests only; not on the data path).
  *   lowdiff_launch_count: number of kernels this library has launched in the process.
  *   lowdiff_profile_enable(1): from now on, bracket every launch of the named kernel classes
  *     with CUDA events on the launching stream; lowdiff_profile_query sums the elapsed time
  *     (synchronizing the events) of launches whose class name equals `name`, then forgets them.
- *     Classes: "compress_stream", "compress_sample", "compress_select", "compress_emit",
- *     "coalesce", "merge", "merge_pack", "replay_dense", "replay_sparse", "starts".
+ *     Classes: "compress_stream", "compress_sample", "compress_select", "coalesce", "merge",
+ *     "merge_pack", "replay_dense", "replay_sparse", "starts".
  * ------------------------------------------------------------------------------------------- */
 uint64_t       lowdiff_launch_count(void);
 /* After a lowdiff_compress on `stream` with workspace `ws` (syncs the stream): out6 = {sampled

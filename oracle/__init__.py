@@ -16,6 +16,8 @@ Functions (numpy in, numpy out) and the passage each follows:
   batch_merge   O3+O4  batched C^B_t, §4.2 Step 2; serialized record bytes
   record_size       record byte-size formula (DESIGN.md §Record layout)
   replay        O5  Recovery, Alg.1 lines 16-24; Adam Eq.1
+  config_model  O6  (module oracle.config_model, plain fp64 Python) Eq. 3 / Eq. 5 of §3.5
+                    (P:318-350): wasted time, (f*, b*), the best integer (FCF, B)
 
 Parity pins for every function are in tests/test_oracle_*.py (none is "parity unpinned").
 """

@@ -77,7 +77,7 @@ EXPORTS = [
     "lowdiff_batch_merge", "lowdiff_record_bytes", "lowdiff_stage_d2h", "lowdiff_record_parse",
     "lowdiff_replay_workspace_size", "lowdiff_replay", "lowdiff_launch_count",
     "lowdiff_profile_enable", "lowdiff_profile_query", "lowdiff_compress_stats",
-    "lowdiff_debug_force_threshold",
+    "lowdiff_debug_force_threshold", "lowdiff_wasted_time", "lowdiff_optimal_config",
 ]
 
 _lib = None
@@ -125,6 +125,8 @@ def lib() -> C.CDLL:
         "lowdiff_profile_query": ([C.c_char_p, vp, vp], i32),
         "lowdiff_compress_stats": ([vp, u64, u64, vp, vp], i32),
         "lowdiff_debug_force_threshold": ([i32, C.c_uint32], i32),
+        "lowdiff_wasted_time": ([vp, f64, f64, vp], i32),
+        "lowdiff_optimal_config": ([vp, vp, vp, vp, vp], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -184,6 +186,33 @@ def shard_bounds(n: int, nranks: int, rank: int) -> tuple[int, int]:
     lo, hi = C.c_uint64(), C.c_uint64()
     _check(lib().lowdiff_shard_bounds(n, nranks, rank, C.byref(lo), C.byref(hi)), "shard_bounds")
     return lo.value, hi.value
+
+
+class ConfigModel(C.Structure):
+    """lowdiff_config_model (§3.5): time in units of one training iteration."""
+    _fields_ = [(k, C.c_double) for k in ("N", "M", "W", "S", "T", "R_F", "R_D")]
+
+
+def _model(m: dict) -> ConfigModel:
+    return ConfigModel(*(float(m[k]) for k in ("N", "M", "W", "S", "T", "R_F", "R_D")))
+
+
+def wasted_time(model: dict, f: float, b: float) -> float:
+    """Eq. 3 for full-checkpoint frequency f and batching size b."""
+    out = C.c_double()
+    cm = _model(model)
+    _check(lib().lowdiff_wasted_time(C.byref(cm), float(f), float(b), C.byref(out)), "wasted_time")
+    return out.value
+
+
+def optimal_config(model: dict) -> dict:
+    """Eq. 5 and the best integer (FCF, B) around it: {"f_star", "b_star", "fcf", "B"}."""
+    fs, bs = C.c_double(), C.c_double()
+    fcf, b = C.c_uint32(), C.c_uint32()
+    cm = _model(model)
+    _check(lib().lowdiff_optimal_config(C.byref(cm), C.byref(fs), C.byref(bs), C.byref(fcf), C.byref(b)),
+           "optimal_config")
+    return {"f_star": fs.value, "b_star": bs.value, "fcf": fcf.value, "B": b.value}
 
 
 def record_size(mode, B: int, nnz: int, nent: int) -> int:
