@@ -222,6 +222,26 @@ lowdiff_status lowdiff_replay(lowdiff_state* st, const lowdiff_opt* opt,
                               uint64_t ws_bytes, lowdiff_stream_t stream);
 
 /* ---------------------------------------------------------------------------------------------
+ * (5b) Parallel recovery — §4.4 "Parallel recovery module" on Eq. 2 (P:92,
+ *     M_n = C^F + C^D_1 + ... + C^D_n): for plain SGD (weight_decay 0) over SUM records that share
+ *     one constant lr, the chain's differentials are first merged among themselves — ONE multiway
+ *     merge (the paper's pairwise tree in a single level): per index, the record-ascending fp32 sum
+ *     of the records' values, absent terms skipped — and the merged differential is applied to the
+ *     checkpoint once:  x[i] = x[i] - lr * (v_1[i] + ... + v_R[i]).  One merge touches C^F instead
+ *     of R. Its rounding differs from lowdiff_replay's sequential
+ *     x - lr v_1 - lr v_2 ...: the two agree within the fp32 tolerance, not bit for bit (the CPU
+ *     oracle's parallel recovery is matched bit for bit).
+ *   Arguments, chain checks and state updates as lowdiff_replay (m/v unused); at most 256 records.
+ *   Errors: as lowdiff_replay; EUNSUPPORTED unless SGD with weight_decay 0, every record SUM and
+ *   every lr[] entry equal.
+ * ------------------------------------------------------------------------------------------- */
+lowdiff_status lowdiff_replay_parallel_workspace_size(const lowdiff_state* st, const lowdiff_record_view* recs,
+                                                      uint32_t nrec, uint64_t* bytes);
+lowdiff_status lowdiff_replay_parallel(lowdiff_state* st, const lowdiff_opt* opt,
+                                       const lowdiff_record_view* recs, uint32_t nrec, void* ws,
+                                       uint64_t ws_bytes, lowdiff_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------------
  * Checkpointing configuration model (§3.5 "Optimizing Checkpointing Configuration", P:318-350;
  * SURVEY §8(f) NEXT-3). Host-only arithmetic (fp64), no stream, no device memory.
  *

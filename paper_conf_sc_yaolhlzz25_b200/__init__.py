@@ -78,6 +78,7 @@ EXPORTS = [
     "lowdiff_replay_workspace_size", "lowdiff_replay", "lowdiff_launch_count",
     "lowdiff_profile_enable", "lowdiff_profile_query", "lowdiff_compress_stats",
     "lowdiff_debug_force_threshold", "lowdiff_wasted_time", "lowdiff_optimal_config",
+    "lowdiff_replay_parallel_workspace_size", "lowdiff_replay_parallel",
 ]
 
 _lib = None
@@ -126,6 +127,8 @@ def lib() -> C.CDLL:
         "lowdiff_compress_stats": ([vp, u64, u64, vp, vp], i32),
         "lowdiff_debug_force_threshold": ([i32, C.c_uint32], i32),
         "lowdiff_wasted_time": ([vp, f64, f64, vp], i32),
+        "lowdiff_replay_parallel_workspace_size": ([vp, vp, C.c_uint32, vp], i32),
+        "lowdiff_replay_parallel": ([vp, vp, vp, C.c_uint32, vp, u64, vp], i32),
         "lowdiff_optimal_config": ([vp, vp, vp, vp, vp], i32),
     }
     for name, (args, res) in sig.items():
@@ -427,10 +430,7 @@ def record_parse(h_bytes) -> dict:
 
 
 # ---- (5) replay ----------------------------------------------------------------------------------------
-def replay(state: dict, opt: dict, records, ws=None, stream=None) -> dict:
-    """Recovery (Alg.1 lines 16-24): replay records [(d_record uint8 CUDA tensor, h_head host bytes)]
-    onto the state {x, m, v (fp32 CUDA), x_bf16 (optional), n, lo, hi, t, adam_step,
-    momentum_initialized}; device arrays are updated in place, counters in the dict."""
+def _replay_args(state: dict, opt: dict, records):
     import numpy as np
     o = Opt(_KIND[opt["kind"]], opt.get("momentum", 0.0), opt.get("dampening", 0.0),
             opt.get("weight_decay", 0.0), opt.get("beta1", 0.9), opt.get("beta2", 0.999),
@@ -453,6 +453,14 @@ def replay(state: dict, opt: dict, records, ws=None, stream=None) -> dict:
             keep.append(a)
             hp, hl = a.ctypes.data, a.size
         views[q] = RecordView(_cuda(drec, "d_record"), hp, hl)
+    return o, st, views, R, keep
+
+
+def replay(state: dict, opt: dict, records, ws=None, stream=None) -> dict:
+    """Recovery (Alg.1 lines 16-24): replay records [(d_record uint8 CUDA tensor, h_head host bytes)]
+    onto the state {x, m, v (fp32 CUDA), x_bf16 (optional), n, lo, hi, t, adam_step,
+    momentum_initialized}; device arrays are updated in place, counters in the dict."""
+    o, st, views, R, keep = _replay_args(state, opt, records)
     b = C.c_uint64()
     _check(lib().lowdiff_replay_workspace_size(C.byref(st), views, R, C.byref(b)), "replay_workspace_size")
     if ws is None:
@@ -461,6 +469,21 @@ def replay(state: dict, opt: dict, records, ws=None, stream=None) -> dict:
                                 _stream(stream)), "replay")
     state["t"], state["adam_step"] = st.t, st.adam_step
     state["momentum_initialized"] = st.momentum_initialized
+    return state
+
+
+def replay_parallel(state: dict, opt: dict, records, ws=None, stream=None) -> dict:
+    """Parallel recovery (Eq. 2): merge the chain's SUM differentials once, apply them to the
+    checkpoint once (plain SGD, constant lr). Same arguments as replay()."""
+    o, st, views, R, keep = _replay_args(state, opt, records)
+    b = C.c_uint64()
+    _check(lib().lowdiff_replay_parallel_workspace_size(C.byref(st), views, R, C.byref(b)),
+           "replay_parallel_workspace_size")
+    if ws is None:
+        ws = workspace(b.value, state["x"].device, "replay_parallel")
+    _check(lib().lowdiff_replay_parallel(C.byref(st), C.byref(o), views, R, _cuda(ws, "ws"), ws.numel(),
+                                         _stream(stream)), "replay_parallel")
+    state["t"] = st.t
     return state
 
 

@@ -443,6 +443,50 @@ lowdiff_status lowdiff_replay(lowdiff_state* st, const lowdiff_opt* opt, const l
   return replay_run(st, opt, R.data(), nrec, ws, (cudaStream_t)stream);
 }
 
+static lowdiff_status parallel_supported(const lowdiff_opt* o, const std::vector<RecInfo>& R) {
+  if (o->kind != LOWDIFF_OPT_SGD || o->weight_decay != 0.0)
+    return fail(LOWDIFF_EUNSUPPORTED, "replay_parallel: plain SGD (weight_decay 0) only");
+  if (R.size() > (size_t)kMaxLists) return fail(LOWDIFF_EUNSUPPORTED, "replay_parallel: more than %d records", kMaxLists);
+  for (const RecInfo& r : R) {
+    if (r.mode != LOWDIFF_MERGE_SUM) return fail(LOWDIFF_EUNSUPPORTED, "replay_parallel: SUM records only");
+    for (uint32_t j = 0; j < r.B; ++j)
+      if (r.h_lr[j] != R[0].h_lr[0]) return fail(LOWDIFF_EUNSUPPORTED, "replay_parallel: lr must be one constant");
+  }
+  return LOWDIFF_OK;
+}
+
+lowdiff_status lowdiff_replay_parallel_workspace_size(const lowdiff_state* st, const lowdiff_record_view* recs,
+                                                      uint32_t nrec, uint64_t* bytes) {
+  if (!st || !bytes || st->lo >= st->hi || (nrec && !recs)) return fail(LOWDIFF_EINVAL, "replay_parallel_workspace_size");
+  uint64_t entries = 0;
+  for (uint32_t q = 0; q < nrec; ++q) {
+    lowdiff_record_header h;
+    lowdiff_status s = lowdiff_record_parse(recs[q].h_head, recs[q].h_head_len, &h);
+    if (s) return s;
+    entries += h.nnz;
+  }
+  *bytes = replay_parallel_ws_bytes(nrec ? nrec : 1, entries, st->lo, st->hi);
+  return LOWDIFF_OK;
+}
+
+lowdiff_status lowdiff_replay_parallel(lowdiff_state* st, const lowdiff_opt* opt, const lowdiff_record_view* recs,
+                                       uint32_t nrec, void* ws, uint64_t ws_bytes, lowdiff_stream_t stream) {
+  lowdiff_status s = check_state(st, opt);
+  if (s) return s;
+  if (nrec && !recs) return fail(LOWDIFF_EINVAL, "replay_parallel: null records");
+  std::vector<RecInfo> R;
+  s = build_recinfo(st, opt, recs, nrec, R);
+  if (s) return s;
+  if (nrec == 0) return LOWDIFF_OK;
+  s = parallel_supported(opt, R);
+  if (s) return s;
+  uint64_t entries = 0;
+  for (const RecInfo& r : R) entries += r.nnz;
+  if (!ws || !aligned16(ws) || ws_bytes < replay_parallel_ws_bytes(nrec, entries, st->lo, st->hi))
+    return fail(LOWDIFF_EWORKSPACE, "replay_parallel: workspace too small");
+  return replay_parallel_run(st, R.data(), nrec, ws, (cudaStream_t)stream);
+}
+
 // ---- instrumentation ------------------------------------------------------------------------------
 uint64_t lowdiff_launch_count(void) { return g_launches.load(); }
 

@@ -77,5 +77,8 @@ struct RecInfo {            // parsed on the host from the record header
 uint64_t replay_ws_bytes(uint64_t len, const RecInfo* recs, uint32_t nrec);
 lowdiff_status replay_run(lowdiff_state* st, const lowdiff_opt* o, const RecInfo* recs,
                           uint32_t nrec, void* ws, cudaStream_t s);
+uint64_t replay_parallel_ws_bytes(uint32_t nrec, uint64_t entries, uint64_t lo, uint64_t hi);
+lowdiff_status replay_parallel_run(lowdiff_state* st, const RecInfo* recs, uint32_t nrec, void* ws,
+                                   cudaStream_t s);
 
 }  // namespace lowdiff
