@@ -222,6 +222,23 @@ lowdiff_status lowdiff_replay(lowdiff_state* st, const lowdiff_opt* opt,
                               uint64_t ws_bytes, lowdiff_stream_t stream);
 
 /* ---------------------------------------------------------------------------------------------
+ * (5c) Live update — Alg.1 training process, "G_t <- Comp^{-1}(G~_t)" and "M_{t+1} <- M_t +
+ *     Adam(o_t, G_t)": the synchronized G~_t of the current iteration, exactly as
+ *     lowdiff_allgather_sparse / lowdiff_coalesce leave it in device memory (idx ascending unique in
+ *     [lo, hi), val fp32, *d_nnz entries, g->cap >= *d_nnz host bound, g->lr this iteration's lr),
+ *     applied to the live shard state in place as ONE dense optimizer step. The arithmetic is that of
+ *     lowdiff_replay on a one-iteration record of G~_t, so a later recovery from the differentials
+ *     reproduces the live trajectory bit for bit (Finding 1). Unlike lowdiff_replay it never
+ *     reads a header on the host and never synchronizes (capturable in a CUDA graph).
+ *   st: as lowdiff_replay; st->t, st->adam_step, st->momentum_initialized advance by one step.
+ *   ws: lowdiff_update_workspace_size bytes, device, 16-byte aligned, caller-owned.
+ * Errors: EINVAL (null pointers, cap > hi - lo, bad state), EWORKSPACE, EUNSUPPORTED (Adam + wd).
+ * ------------------------------------------------------------------------------------------- */
+lowdiff_status lowdiff_update_workspace_size(const lowdiff_state* st, uint64_t* bytes);
+lowdiff_status lowdiff_update(lowdiff_state* st, const lowdiff_opt* opt, const lowdiff_diff_view* g,
+                              void* ws, uint64_t ws_bytes, lowdiff_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------------
  * (5b) Parallel recovery — §4.4 "Parallel recovery module" on Eq. 2 (P:92,
  *     M_n = C^F + C^D_1 + ... + C^D_n): for plain SGD (weight_decay 0) over SUM records that share
  *     one constant lr, the chain's differentials are first merged among themselves — ONE multiway

@@ -79,6 +79,7 @@ EXPORTS = [
     "lowdiff_profile_enable", "lowdiff_profile_query", "lowdiff_compress_stats",
     "lowdiff_debug_force_threshold", "lowdiff_wasted_time", "lowdiff_optimal_config",
     "lowdiff_replay_parallel_workspace_size", "lowdiff_replay_parallel",
+    "lowdiff_update_workspace_size", "lowdiff_update",
 ]
 
 _lib = None
@@ -130,6 +131,8 @@ def lib() -> C.CDLL:
         "lowdiff_replay_parallel_workspace_size": ([vp, vp, C.c_uint32, vp], i32),
         "lowdiff_replay_parallel": ([vp, vp, vp, C.c_uint32, vp, u64, vp], i32),
         "lowdiff_optimal_config": ([vp, vp, vp, vp, vp], i32),
+        "lowdiff_update_workspace_size": ([vp, vp], i32),
+        "lowdiff_update": ([vp, vp, vp, vp, u64, vp], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -467,6 +470,25 @@ def replay(state: dict, opt: dict, records, ws=None, stream=None) -> dict:
         ws = workspace(b.value, state["x"].device, "replay")
     _check(lib().lowdiff_replay(C.byref(st), C.byref(o), views, R, _cuda(ws, "ws"), ws.numel(),
                                 _stream(stream)), "replay")
+    state["t"], state["adam_step"] = st.t, st.adam_step
+    state["momentum_initialized"] = st.momentum_initialized
+    return state
+
+
+def update(state: dict, opt: dict, g_t, ws=None, stream=None) -> dict:
+    """Live update (Alg.1 training process): apply this iteration's synchronized G~_t =
+    (idx int32, val fp32, d_nnz int64[1], cap, lr) — as allgather_sparse/coalesce return it — to the
+    state as one dense optimizer step, in place, without a host synchronization. Bit-identical to
+    replay() of a one-iteration record of G~_t."""
+    o, st, _, _, _ = _replay_args(state, opt, [])
+    idx, val, d_nnz, cap, lr = g_t
+    view = DiffView(_cuda(idx, "idx"), _cuda(val, "val"), _cuda(d_nnz, "d_nnz"), int(cap), float(lr))
+    b = C.c_uint64()
+    _check(lib().lowdiff_update_workspace_size(C.byref(st), C.byref(b)), "update_workspace_size")
+    if ws is None:
+        ws = workspace(b.value, state["x"].device, "update")
+    _check(lib().lowdiff_update(C.byref(st), C.byref(o), C.byref(view), _cuda(ws, "ws"), ws.numel(),
+                                _stream(stream)), "update")
     state["t"], state["adam_step"] = st.t, st.adam_step
     state["momentum_initialized"] = st.momentum_initialized
     return state

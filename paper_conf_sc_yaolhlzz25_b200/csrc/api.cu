@@ -443,6 +443,33 @@ lowdiff_status lowdiff_replay(lowdiff_state* st, const lowdiff_opt* opt, const l
   return replay_run(st, opt, R.data(), nrec, ws, (cudaStream_t)stream);
 }
 
+lowdiff_status lowdiff_update_workspace_size(const lowdiff_state* st, uint64_t* bytes) {
+  if (!st || !bytes || st->lo >= st->hi) return fail(LOWDIFF_EINVAL, "update_workspace_size");
+  *bytes = replay_ws_bytes(st->hi - st->lo, nullptr, 1) + 256;
+  return LOWDIFF_OK;
+}
+
+lowdiff_status lowdiff_update(lowdiff_state* st, const lowdiff_opt* opt, const lowdiff_diff_view* g, void* ws,
+                              uint64_t ws_bytes, lowdiff_stream_t stream) {
+  lowdiff_status s = check_state(st, opt);
+  if (s) return s;
+  if (!g || !g->idx || !g->val || !g->d_nnz) return fail(LOWDIFF_EINVAL, "update: null gradient view");
+  if (g->cap > st->hi - st->lo) return fail(LOWDIFF_EINVAL, "update: cap exceeds the shard length");
+  RecInfo r;                                       // G~_t as a one-iteration SUM list (count on device)
+  r.d = nullptr;
+  r.mode = LOWDIFF_MERGE_SUM;
+  r.B = 1;
+  r.nnz = r.nent = g->cap;
+  r.off_lr = r.off_idx = r.off_val = r.off_off = r.off_it = 0;
+  r.h_lr = &g->lr;
+  r.live_idx = g->idx;
+  r.live_val = g->val;
+  r.d_nnz = g->d_nnz;
+  if (!ws || !aligned16(ws) || ws_bytes < replay_ws_bytes(st->hi - st->lo, &r, 1))
+    return fail(LOWDIFF_EWORKSPACE, "update: workspace too small");
+  return replay_run(st, opt, &r, 1, ws, (cudaStream_t)stream);
+}
+
 static lowdiff_status parallel_supported(const lowdiff_opt* o, const std::vector<RecInfo>& R) {
   if (o->kind != LOWDIFF_OPT_SGD || o->weight_decay != 0.0)
     return fail(LOWDIFF_EUNSUPPORTED, "replay_parallel: plain SGD (weight_decay 0) only");

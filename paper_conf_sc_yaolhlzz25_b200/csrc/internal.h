@@ -73,6 +73,11 @@ struct RecInfo {            // parsed on the host from the record header
   uint64_t nnz, nent;
   uint64_t off_lr, off_idx, off_val, off_off, off_it;   // section byte offsets
   const float* h_lr;        // host lr[B]
+  // live update (lowdiff_update): a bare (idx, val) list whose length lives on the device; then
+  // d == nullptr, mode == SUM, B == 1 and nnz is the host upper bound (cap)
+  const uint32_t* live_idx = nullptr;
+  const float* live_val = nullptr;
+  const uint64_t* d_nnz = nullptr;
 };
 uint64_t replay_ws_bytes(uint64_t len, const RecInfo* recs, uint32_t nrec);
 lowdiff_status replay_run(lowdiff_state* st, const lowdiff_opt* o, const RecInfo* recs,

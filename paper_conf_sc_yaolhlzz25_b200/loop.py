@@ -2,19 +2,25 @@
 dependency analysis of §3.4): the compressed, synchronized gradient G~_t of every
 training iteration both drives the live optimizer update and IS the differential checkpoint.
 
-Per iteration t (one call of `LowDiffLoop.step(grad)`):
+Per iteration t (one call of `LowDiffLoop.step(grad)`), all on the training stream, no host sync:
   1. G~_t <- Sync(Comp(G_t))        lowdiff_compress (top-k + EF) -> lowdiff_allgather_sparse
-  2. live update M_{t+1} = M_t + Opt(G~_t) on this rank's shard: G~_t as a one-iteration record
-     (lowdiff_batch_merge, STACK) replayed onto the live state (lowdiff_replay, K = 1) — the
-     same kernels and op order recovery uses, so recovery reproduces the live trajectory bit for
-     bit (Finding 1)
-  3. the Reusing Queue: G~_t is handed to the checkpoint side without a copy of its
-     values through the device ring; every B iterations the batch is merged into one record and
-     staged to pinned host memory on a copy stream (§4.2)
-  4. every `full_every` iterations (and at t = 0) a full checkpoint C^F_t of the shard state.
+  2. live update M_{t+1} = M_t + Opt(G~_t) on this rank's shard: lowdiff_update — the replay
+     kernel on G~_t as a one-iteration differential, so recovery reproduces the live trajectory
+     bit for bit (Finding 1)
+  3. the Reusing Queue: G~_t stays in its own ring slot (no copy of its values); every
+     B iterations the batch is merged into one record on the training stream (§4.2)
+     into one of two device record buffers
+  4. the checkpoint side (`_service`, run by the host at the start of each step): once a merge has
+     finished (event query, never a wait) the record's byte count is read from pinned memory and
+     the record is staged D2H on a copy stream into a pinned buffer from a reused pool (the
+     paper's offload_to_cpu)
+  5. every `full_every` iterations (and at t = 0) a full checkpoint C^F_t: a device snapshot of
+     the shard state (D2D on the training stream), then D2H on the copy stream (CheckFreq-style
+     snapshot -> persist). Older full checkpoints and the records before them are
+     released once a newer full checkpoint is on the host (`retain_fulls`; None keeps all).
 
 `recover(t)` rebuilds the state at iteration t from the latest full checkpoint at or before t
-and the staged records after it (Alg. 1 lines 16-24), through lowdiff_replay.
+and the staged records after it (Alg. 1 lines 16-24): host -> device loads, then lowdiff_replay.
 
 Marshalling only: every step runs in liblowdiff's kernels (or NCCL); this module owns buffers,
 streams and bookkeeping.
@@ -24,95 +30,200 @@ from __future__ import annotations
 import numpy as np
 import torch
 
-from . import (allgather_sparse, batch_merge, compress, k_for_density, record_bytes, replay,
-               shard_bounds, stage_d2h)
+from . import (LowDiffError, allgather_sparse, batch_merge, compress, k_for_density, pairs_bytes,
+               record_max_bytes, replay, shard_bounds, stage_d2h, update)
+
+_STATE_KEYS = ("x", "m", "v")
 
 
 class LowDiffLoop:
     def __init__(self, x: torch.Tensor, opt: dict, lr: float, rho: float, B: int, full_every: int,
-                 comm=None, rank: int = 0, world: int = 1, adam_step: int = 0, checkpoint: bool = True):
+                 comm=None, rank: int = 0, world: int = 1, adam_step: int = 0, checkpoint: bool = True,
+                 retain_fulls: int | None = 2):
         assert x.dtype == torch.float32 and x.is_cuda and x.dim() == 1
         assert full_every % B == 0, "full checkpoints fall on batch boundaries (records chain from them)"
+        assert retain_fulls is None or retain_fulls >= 1
         self.n = x.numel()
         self.k = k_for_density(self.n, rho)
         self.lo, self.hi = shard_bounds(self.n, world, rank)
         self.world, self.comm, self.opt = world, comm, dict(opt)
         self.lr = float(np.float32(lr))
-        self.B, self.full_every = B, full_every
-        self.r = torch.zeros(self.n, device=x.device)                 # EF residual
+        self.B, self.full_every, self.retain_fulls = B, full_every, retain_fulls
+        dev = x.device
+        self.r = torch.zeros(self.n, device=dev)                      # EF residual
         L = self.hi - self.lo
         kind = opt["kind"]
-        self.state = {"x": x[self.lo:self.hi], "m": None if kind == "sgd" else torch.zeros(L, device=x.device),
-                      "v": torch.zeros(L, device=x.device) if kind == "adam" else None, "x_bf16": None,
+        self.state = {"x": x[self.lo:self.hi], "m": None if kind == "sgd" else torch.zeros(L, device=dev),
+                      "v": torch.zeros(L, device=dev) if kind == "adam" else None, "x_bf16": None,
                       "n": self.n, "lo": self.lo, "hi": self.hi, "t": 0, "adam_step": adam_step,
                       "momentum_initialized": 0}
         self.cap = min(world * self.k, L)
-        self.ring = []                                                  # G~ of the open batch
-        self.records = []                                               # (t_first, device rec, pinned)
-        self.fulls = []                                                 # (t, {x, m, v, adam_step, mi})
-        self.copy_stream = torch.cuda.Stream(device=x.device)
         self.checkpoint = checkpoint          # False: the same training step without checkpointing
         self.t = 0
+        self.copy_stream = torch.cuda.Stream(device=dev)
+        # the Reusing Queue: B ring slots of G~ (the open batch). The batch merge is issued on the
+        # training stream right after the batch's last update, so stream order puts it before the
+        # next batch's writes into the same slots.
+        R = B if checkpoint else 1
+        self.slots = [(torch.empty(self.cap, dtype=torch.int32, device=dev),
+                       torch.empty(self.cap, dtype=torch.float32, device=dev),
+                       torch.zeros(1, dtype=torch.int64, device=dev)) for _ in range(R)]
+        self.ring = []                                                  # G~ of the open batch
+        self.pairs = torch.empty(pairs_bytes(self.k), dtype=torch.uint8, device=dev)
+        if not checkpoint:
+            return
+        self.rec_cap = record_max_bytes("stack", B, max(B * self.cap, 1))
+        # two device record buffers: one being merged while the other is staged
+        self.drec = [{"buf": torch.empty(self.rec_cap, dtype=torch.uint8, device=dev),
+                      "nb": torch.zeros(1, dtype=torch.int64, device=dev),
+                      "h_nb": torch.zeros(1, dtype=torch.int64, pin_memory=True),
+                      "merged": None, "staged": None, "t_first": None} for _ in range(2)]
+        self.next_drec = 0
+        self.pending = []                                               # merged, not yet staged
+        self.pool = []                                                  # free pinned record buffers
+        self.records = []                                               # (t_first, pinned, nb, copied ev)
+        self.snap = None                                                # device snapshot buffers
+        self.snap_free = None                                           # event: snapshot D2H done
+        self.fulls = []                                                 # (t, {x,m,v pinned,...}, ev)
+        self.full_pool = []                                             # free pinned full buffers
+        if retain_fulls is not None:                                    # reserve the host memory up front
+            L = self.hi - self.lo
+            keys = [k for k in _STATE_KEYS if self.state[k] is not None]
+            self.full_pool = [{k: torch.empty(L, dtype=torch.float32, pin_memory=True) for k in keys}
+                              for _ in range(retain_fulls + 1)]
+            self.pool = [torch.empty(self.rec_cap, dtype=torch.uint8, pin_memory=True)
+                         for _ in range(retain_fulls * (full_every // B) + 2)]
 
     # ---- one training iteration ---------------------------------------------------------------
     def step(self, grad: torch.Tensor):
-        if self.checkpoint and self.t % self.full_every == 0:
-            self._full_checkpoint()
-        pairs = compress(grad, self.r, self.k)
-        idx, val, nnz = allgather_sparse(self.comm, pairs, self.k, "f32", self.lo, self.hi)
+        if self.checkpoint:
+            self._service()
+            if self.t % self.full_every == 0:
+                self._full_checkpoint()
+        idx, val, nnz = self.slots[self.t % len(self.slots)]
+        pairs = compress(grad, self.r, self.k, pairs=self.pairs)
+        allgather_sparse(self.comm, pairs, self.k, "f32", self.lo, self.hi, out_idx=idx, out_val=val,
+                         d_nnz=nnz)
         g_t = (idx, val, nnz, self.cap, self.lr)
-        # live update: G~_t as a one-iteration record, replayed onto the live state (K = 1)
-        rec1, d_nb = batch_merge([g_t], "stack", self.n, self.lo, self.hi, self.t, self.world)
-        nb = record_bytes(d_nb, rec1.numel())
-        head = torch.empty(80 + 4 + 16, dtype=torch.uint8, pin_memory=True)
-        stage_d2h(rec1, 84, head)
-        torch.cuda.current_stream().synchronize()
-        replay(self.state, self.opt, [(rec1[:nb], head)])
+        update(self.state, self.opt, g_t)                               # live M_{t+1}
         self.t += 1
         if not self.checkpoint:
             return
-        # checkpoint side: the ring holds G~_t (its own buffers) until the batch is merged
-        self.ring.append(g_t)
+        self.ring.append(g_t)                                           # Q.put: zero copy
         if len(self.ring) == self.B:
             self._close_batch()
 
     def _close_batch(self):
+        d = self.drec[self.next_drec]
+        self.next_drec ^= 1
+        if d["t_first"] is not None:                                    # buffer still in use
+            self._drain(d)
         t_first = self.t - len(self.ring)
-        rec, d_nb = batch_merge(self.ring, "stack", self.n, self.lo, self.hi, t_first, self.world)
-        nb = record_bytes(d_nb, rec.numel())
-        pinned = torch.empty(nb, dtype=torch.uint8, pin_memory=True)
-        self.copy_stream.wait_stream(torch.cuda.current_stream())
-        stage_d2h(rec, nb, pinned, self.copy_stream)                  # async persist staging
-        self.records.append((t_first, rec, pinned))
+        batch_merge(self.ring, "stack", self.n, self.lo, self.hi, t_first, self.world, record=d["buf"],
+                    d_record_bytes=d["nb"])
+        d["h_nb"].copy_(d["nb"], non_blocking=True)
+        d["merged"] = torch.cuda.Event()
+        d["merged"].record()
+        d["t_first"] = t_first
+        self.pending.append(d)
         self.ring = []
+
+    def _stage(self, d):
+        """Checkpoint side: the merge of `d` has finished; stage its bytes to a pinned buffer."""
+        nb = int(d["h_nb"][0])
+        if nb > self.rec_cap:
+            raise LowDiffError(4, f"record of {nb} bytes exceeds its buffer ({self.rec_cap})")
+        pinned = self.pool.pop() if self.pool else torch.empty(self.rec_cap, dtype=torch.uint8, pin_memory=True)
+        self.copy_stream.wait_event(d["merged"])
+        stage_d2h(d["buf"], nb, pinned, self.copy_stream)
+        ev = torch.cuda.Event()
+        ev.record(self.copy_stream)
+        d["staged"] = ev
+        self.records.append((d["t_first"], pinned, nb, ev))
+        self.pending = [p for p in self.pending if p is not d]
+
+    def _drain(self, d):
+        if any(p is d for p in self.pending):
+            d["merged"].synchronize()
+            self._stage(d)
+        d["staged"].synchronize()
+        d["t_first"] = None
+
+    def _service(self):
+        for d in list(self.pending):
+            if d["merged"].query():
+                self._stage(d)
+        self._retire()
+
+    def _retire(self):
+        """Release full checkpoints (and the records before them) older than the newest
+        `retain_fulls` full checkpoints that are completely on the host."""
+        if self.retain_fulls is None:
+            return
+        done = [f for f in self.fulls if f[2].query()]
+        if len(done) < self.retain_fulls:
+            return
+        t_keep = done[-self.retain_fulls][0]
+        for f in self.fulls:
+            if f[0] < t_keep:
+                self.full_pool.append({k: f[1][k] for k in _STATE_KEYS if k in f[1]})
+        self.fulls = [f for f in self.fulls if f[0] >= t_keep]
+        keep = []
+        for rec in self.records:
+            if rec[0] < t_keep and rec[3].query():
+                self.pool.append(rec[1])
+            else:
+                keep.append(rec)
+        self.records = keep
 
     def _full_checkpoint(self):
         st = self.state
-        snap = {"x": st["x"].clone(), "m": None if st["m"] is None else st["m"].clone(),
-                "v": None if st["v"] is None else st["v"].clone(), "adam_step": st["adam_step"],
-                "momentum_initialized": st["momentum_initialized"]}
-        self.fulls.append((self.t, snap))
+        if self.snap is None:
+            self.snap = {k: torch.empty_like(st[k]) for k in _STATE_KEYS if st[k] is not None}
+        elif self.snap_free is not None:
+            self.snap_free.synchronize()                                # previous D2H finished
+        for k, buf in self.snap.items():                                # snapshot (training stream)
+            buf.copy_(st[k])
+        taken = torch.cuda.Event()
+        taken.record()
+        self.copy_stream.wait_event(taken)
+        host = self.full_pool.pop() if self.full_pool else \
+            {k: torch.empty(buf.numel(), dtype=buf.dtype, pin_memory=True) for k, buf in self.snap.items()}
+        with torch.cuda.stream(self.copy_stream):                       # persist (copy engine)
+            for k, buf in self.snap.items():
+                host[k].copy_(buf, non_blocking=True)
+        ev = torch.cuda.Event()
+        ev.record(self.copy_stream)
+        self.snap_free = ev
+        host.update(adam_step=st["adam_step"], momentum_initialized=st["momentum_initialized"])
+        self.fulls.append((self.t, host, ev))
+
+    def flush(self):
+        """Wait until every closed batch and full checkpoint is on the host."""
+        for d in list(self.pending):
+            d["merged"].synchronize()
+            self._stage(d)
+        self.copy_stream.synchronize()
 
     # ---- recovery (Alg. 1 lines 16-24) -----------------------------------------------------------
     def recover(self, t: int) -> dict:
         """State of this shard at iteration t (t a batch boundary), from the latest full checkpoint
-        at or before t and the staged records after it."""
-        self.copy_stream.synchronize()
-        tf, snap = max((f for f in self.fulls if f[0] <= t), key=lambda f: f[0])
-        L = self.hi - self.lo
-        st = {"x": torch.empty(L, device=snap["x"].device), "x0": snap["x"],
-              "m": None if snap["m"] is None else torch.empty_like(snap["m"]), "m0": snap["m"],
-              "v": None if snap["v"] is None else torch.empty_like(snap["v"]), "v0": snap["v"],
+        at or before t and the staged records after it, loaded back from the host."""
+        self.flush()
+        tf, snap, _ = max((f for f in self.fulls if f[0] <= t), key=lambda f: f[0])
+        dev = self.state["x"].device
+        load = lambda k: None if k not in snap else snap[k].to(dev, non_blocking=True)
+        st = {"x": torch.empty(self.hi - self.lo, device=dev), "x0": load("x"),
+              "m": None if "m" not in snap else torch.empty_like(snap["m"], device=dev), "m0": load("m"),
+              "v": None if "v" not in snap else torch.empty_like(snap["v"], device=dev), "v0": load("v"),
               "x_bf16": None, "n": self.n, "lo": self.lo, "hi": self.hi, "t": tf,
               "adam_step": snap["adam_step"], "momentum_initialized": snap["momentum_initialized"]}
-        chain = [(rec, pinned) for (t0, rec, pinned) in self.records if tf <= t0 < t]
+        chain = sorted((r for r in self.records if tf <= r[0] < t), key=lambda r: r[0])
         if chain:
-            replay(st, self.opt, [(rec[:p.numel()], p) for rec, p in chain])
+            replay(st, self.opt, [(p[:nb].to(dev, non_blocking=True), p[:nb]) for _, p, nb, _ in chain])
         else:
-            st["x"].copy_(snap["x"])
-            if st["m"] is not None:
-                st["m"].copy_(snap["m"])
-            if st["v"] is not None:
-                st["v"].copy_(snap["v"])
+            for k in _STATE_KEYS:
+                if st[k] is not None:
+                    st[k].copy_(st[k + "0"])
         assert st["t"] == t, (st["t"], t)
         return st
