@@ -380,11 +380,19 @@ def run_ours(args, cfg):
                        "achieved_gbs": alg / t_s / 1e9, "hbm_frac": alg / t_s / 1e9 / hbm_peak,
                        "ms_per_step": rp_ms / args.steps}
         if cfg.opt == "adam":
-            # 2 MUFU ops (rsqrt, rcp) per parameter-step at 16/clk/SM on 148 SMs
+            # Per parameter-step the exact Adam step issues 15 fp32 operations (FFMA2 pairs) and 2
+            # MUFU ops. Measured on B200 (scripts/micro/adam_mix.cu, profiles/adam_mix_r01.txt):
+            # fp32 128 lanes/clk/SM, MUFU 32/clk/SM, so the fp32 pipe is the floor; the same
+            # instruction mix with no memory or bookkeeping peaks at 1.96 T parameter-steps/s.
             f_mhz = (clk or {}).get("sm_mhz") or 1965.0
-            floor_s = 2.0 * nloc * R * B / (148 * 16 * f_mhz * 1e6)
+            psteps = nloc * R * B
+            floor_s = 15.0 * psteps / (148 * 128 * f_mhz * 1e6)
+            mix_s = psteps / 1.96e12
             replay_roof.update({"bound": "alu", "alu_floor_ms": floor_s * 1e3, "alu_frac": floor_s / t_s,
-                                "alu_peak": f"MUFU 16/clk/SM x 148 SMs at {f_mhz:.0f} MHz"})
+                                "alu_peak": f"fp32 128 lanes/clk/SM x 148 SMs at {f_mhz:.0f} MHz (15 ops per "
+                                            "parameter-step; MUFU 32/clk/SM is not binding)",
+                                "mix_ceiling_ms": mix_s * 1e3, "mix_frac": mix_s / t_s,
+                                "param_steps_per_s": psteps / t_s})
         else:
             replay_roof["bound"] = "alu" if replay_roof["hbm_frac"] < 0.5 else "hbm"
 
