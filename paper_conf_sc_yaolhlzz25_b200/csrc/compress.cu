@@ -198,6 +198,51 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(const void* g, const f
   }
 }
 
+// End of a streaming tile (both stream kernels): the tile's candidates go to the buffer (if it has
+// room) and the residual is stored. A candidate that was recorded is stored as if it were selected
+// (r = 0, or a - fp32(bf16(a)) for bf16 values, reading #8): the select kernel then writes r = a
+// back only for the candidates it rejects (~0.3 k), instead of scattering the k selected ones
+// (a scattered 4-byte store costs a 32-byte DRAM read-modify-write).
+__device__ __forceinline__ float selected_residual(float a, int vbf16) {
+  return vbf16 ? a - __bfloat162float(__float2bfloat16_rn(a)) : 0.0f;
+}
+__device__ __forceinline__ void tile_tail(float (&a)[4][4], uint32_t flags, uint32_t total,
+                                          const uint32_t (&vec_base)[4], uint64_t excl, uint32_t b,
+                                          uint32_t cap, uint64_t base, uint64_t n, bool full, int vbf16,
+                                          float* __restrict__ r, uint32_t* __restrict__ cand_idx,
+                                          float* __restrict__ cand_val) {
+  const int tid = threadIdx.x;
+  const bool rec = total && (uint64_t)b + total <= cap;
+  if (rec && flags) {
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+      uint32_t pos = b + vec_base[c] + (uint32_t)((excl >> (16 * c)) & 0xFFFF);
+#pragma unroll
+      for (int e = 0; e < 4; ++e)
+        if (flags & (1u << (c * 4 + e))) {
+          cand_idx[pos] = (uint32_t)(base + c * 1024 + tid * 4 + e);
+          cand_val[pos] = a[c][e];
+          ++pos;
+        }
+    }
+  }
+  const uint32_t sel = rec ? flags : 0u;
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    float o[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) o[e] = (sel >> (c * 4 + e)) & 1u ? selected_residual(a[c][e], vbf16) : a[c][e];
+    const uint64_t i = base + c * 1024 + tid * 4;
+    if (full) {
+      __stcs(reinterpret_cast<float4*>(r + i), make_float4(o[0], o[1], o[2], o[3]));
+    } else {
+#pragma unroll
+      for (int e = 0; e < 4; ++e)
+        if (i + e < n) r[i + e] = o[e];
+    }
+  }
+}
+
 // ---- K1b: the fused streaming pass ----------------------------------------------------------
 template <bool BF16>
 __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict__ g,
@@ -205,7 +250,8 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
                                                           uint32_t num_tiles, Ctl* ctl,
                                                           uint2* __restrict__ tile_info,
                                                           uint32_t* __restrict__ cand_idx,
-                                                          float* __restrict__ cand_val, uint32_t cap) {
+                                                          float* __restrict__ cand_val, uint32_t cap,
+                                                          int vbf16) {
   __shared__ uint64_t s_scan[2][kThreads / 32];
   __shared__ uint32_t s_base[2];
   const uint32_t T = ctl->t_est;
@@ -227,8 +273,6 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
       for (int c = 0; c < 4; ++c) {
         a[c][0] = gv[c].x + rv[c].x; a[c][1] = gv[c].y + rv[c].y;
         a[c][2] = gv[c].z + rv[c].z; a[c][3] = gv[c].w + rv[c].w;
-        __stcs(reinterpret_cast<float4*>(r + base + c * 1024 + tid * 4),
-               make_float4(a[c][0], a[c][1], a[c][2], a[c][3]));
 #pragma unroll
         for (int e = 0; e < 4; ++e) flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
       }
@@ -241,7 +285,6 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
           a[c][e] = 0.f;
           if (i < n) {
             a[c][e] = load_g1<BF16>(g, i) + r[i];
-            r[i] = a[c][e];
             flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
           }
         }
@@ -275,22 +318,8 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
       tile_info[tile] = make_uint2(b, total);
     }
     __syncthreads();
-    if (total) {
-      const uint32_t b = s_base[par];
-      if ((uint64_t)b + total <= cap && flags) {
-#pragma unroll
-        for (int c = 0; c < 4; ++c) {
-          uint32_t pos = b + vec_base[c] + (uint32_t)((excl >> (16 * c)) & 0xFFFF);
-#pragma unroll
-          for (int e = 0; e < 4; ++e)
-            if (flags & (1u << (c * 4 + e))) {
-              cand_idx[pos] = (uint32_t)(base + c * 1024 + tid * 4 + e);
-              cand_val[pos] = a[c][e];
-              ++pos;
-            }
-        }
-      }
-    }
+    tile_tail(a, flags, total, vec_base, excl, s_base[par], cap, base, n, base + kTile <= n, vbf16, r,
+              cand_idx, cand_val);
   }
 }
 
@@ -309,7 +338,8 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
                                                               uint32_t num_tiles, Ctl* ctl,
                                                               uint2* __restrict__ tile_info,
                                                               uint32_t* __restrict__ cand_idx,
-                                                              float* __restrict__ cand_val, uint32_t cap) {
+                                                              float* __restrict__ cand_val, uint32_t cap,
+                                                              int vbf16) {
   constexpr uint32_t kGB = kTile * (BF16 ? 2 : 4), kRB = kTile * 4, kSB = kGB + kRB;
   extern __shared__ __align__(128) uint8_t s_tiles[];          // kStages x {g tile, r tile}
   __shared__ __align__(8) uint64_t s_bar[kStages];
@@ -370,18 +400,9 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
 #pragma unroll
     for (int c = 0; c < 4; ++c) {
       const uint64_t i = base + c * 1024 + tid * 4;
-      if (tile < full_tiles) {
-        __stcs(reinterpret_cast<float4*>(r + i), make_float4(a[c][0], a[c][1], a[c][2], a[c][3]));
 #pragma unroll
-        for (int e = 0; e < 4; ++e) flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
-      } else {
-#pragma unroll
-        for (int e = 0; e < 4; ++e)
-          if (i + e < n) {
-            r[i + e] = a[c][e];
-            flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
-          }
-      }
+      for (int e = 0; e < 4; ++e)
+        if (tile < full_tiles || i + e < n) flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
     }
     // Order-preserving compaction: one block scan of 4 x 16-bit per-vector counts.
     uint64_t packed = 0;
@@ -416,22 +437,8 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
       tile_info[tile] = make_uint2(b, total);
     }
     __syncthreads();
-    if (total) {
-      const uint32_t b = s_base[par];
-      if ((uint64_t)b + total <= cap && flags) {
-#pragma unroll
-        for (int c = 0; c < 4; ++c) {
-          uint32_t pos = b + vec_base[c] + (uint32_t)((excl >> (16 * c)) & 0xFFFF);
-#pragma unroll
-          for (int e = 0; e < 4; ++e)
-            if (flags & (1u << (c * 4 + e))) {
-              cand_idx[pos] = (uint32_t)(base + c * 1024 + tid * 4 + e);
-              cand_val[pos] = a[c][e];
-              ++pos;
-            }
-        }
-      }
-    }
+    tile_tail(a, flags, total, vec_base, excl, s_base[par], cap, base, n, tile < full_tiles, vbf16, r,
+              cand_idx, cand_val);
   }
 }
 
@@ -531,6 +538,17 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
   const uint32_t mode = (cc >= k && cc <= cap) ? 0u : 1u;
   const float* src = mode ? r : cand_val;
   const uint64_t N = mode ? n : (uint64_t)cc;
+  if (mode) {
+    // full-array fallback: the stream pass stored the recorded candidates' residual as if they
+    // were selected; put a = g + r back for them first (their values are in the buffer)
+    const uint64_t stride = (uint64_t)gridDim.x * kThreads;
+    for (uint64_t t = (uint64_t)blockIdx.x * kThreads + threadIdx.x; t < num_tiles; t += stride) {
+      const uint2 ti = tile_info[t];
+      if (ti.y && (uint64_t)ti.x + ti.y <= cap)
+        for (uint32_t j = 0; j < ti.y; ++j) r[cand_idx[ti.x + j]] = cand_val[ti.x + j];
+    }
+    grid.sync();
+  }
   uint32_t prefix = 0;
   uint64_t need = k;
   select_pass<0>(src, N, sh, h0, prefix, need, s_scan, grid);
@@ -631,11 +649,13 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
         if constexpr (VBF16) {
           const __nv_bfloat16 h = __float2bfloat16_rn(a);
           reinterpret_cast<__nv_bfloat16*>(out_val)[pos] = h;
-          r[idx] = a - __bfloat162float(h);        // exact (Sterbenz), reading #8
+          if (mode) r[idx] = a - __bfloat162float(h);   // exact (Sterbenz), reading #8
         } else {
           reinterpret_cast<float*>(out_val)[pos] = a;
-          r[idx] = 0.0f;
+          if (mode) r[idx] = 0.0f;
         }
+      } else if (in && !mode) {
+        r[idx] = a;                                // a rejected candidate keeps all of a
       }
       gtb += __popc(bg);
       eqb += __popc(be);
@@ -726,6 +746,7 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   uint32_t* cidx = reinterpret_cast<uint32_t*>(w + L.cand_idx);
   float* cval = reinterpret_cast<float*>(w + L.cand_val);
   const bool bf = gdt == LOWDIFF_BF16;
+  const int vbf = vdt == LOWDIFF_BF16 ? 1 : 0;
   static int use_tma = -1;
   if (use_tma < 0) {
     const char* e = getenv("LOWDIFF_STREAM_TMA");
@@ -737,19 +758,19 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
     const int smem = stream_tma_smem(bf);
     if (bf)
       LD_LAUNCH("compress_stream", s, stream_tma_kernel<true>, grid, kThreads, smem, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf);
     else
       LD_LAUNCH("compress_stream", s, stream_tma_kernel<false>, grid, kThreads, smem, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf);
   } else {
     int grid = stream_blocks(bf);
     if ((uint32_t)grid > L.num_tiles) grid = (int)L.num_tiles;
     if (bf)
       LD_LAUNCH("compress_stream", s, stream_kernel<true>, grid, kThreads, 0, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf);
     else
       LD_LAUNCH("compress_stream", s, stream_kernel<false>, grid, kThreads, 0, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf);
   }
 
   {
