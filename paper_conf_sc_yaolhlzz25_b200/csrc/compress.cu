@@ -45,7 +45,7 @@ struct __align__(256) Ctl {
 };
 
 struct Layout {
-  uint64_t ctl, hs, h0, h1, h2, zero_end, tiles, cand_idx, cand_val, tloc, boff, total;
+  uint64_t ctl, hs, hc, h0, h1, h2, zero_end, tiles, cand_idx, cand_val, tloc, boff, total;
   uint32_t num_tiles, cap;
 };
 
@@ -57,6 +57,7 @@ Layout layout(uint64_t n, uint64_t k) {
   uint64_t o = 0;
   L.ctl = o;      o += align256(sizeof(Ctl));
   L.hs = o;       o += align256(4u * bins(0));
+  L.hc = o;       o += align256(4u * bins(0));   // candidates' first digit (stream pass)
   L.h0 = o;       o += align256(4u * bins(0));
   L.h1 = o;       o += align256(4u * bins(1));
   L.h2 = o;       o += align256(4u * bins(2));
@@ -251,9 +252,11 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
                                                           uint2* __restrict__ tile_info,
                                                           uint32_t* __restrict__ cand_idx,
                                                           float* __restrict__ cand_val, uint32_t cap,
-                                                          int vbf16) {
+                                                          int vbf16, uint32_t* __restrict__ hc) {
   __shared__ uint64_t s_scan[2][kThreads / 32];
   __shared__ uint32_t s_base[2];
+  __shared__ uint32_t s_h[bins(0)];               // first-digit histogram of this CTA's candidates
+  for (int j = threadIdx.x; j < bins(0); j += kThreads) s_h[j] = 0;
   const uint32_t T = ctl->t_est;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   int par = 0;
@@ -289,6 +292,13 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
           }
         }
     }
+    if (flags) {                                   // the select's first digit, for free
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          if ((flags >> (c * 4 + e)) & 1u) atomicAdd(&s_h[mag_key(a[c][e]) >> shift(0)], 1u);
+    }
     // Order-preserving compaction: one block scan of 4 x 16-bit per-vector counts.
     uint64_t packed = 0;
 #pragma unroll
@@ -321,6 +331,9 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
     tile_tail(a, flags, total, vec_base, excl, s_base[par], cap, base, n, base + kTile <= n, vbf16, r,
               cand_idx, cand_val);
   }
+  __syncthreads();
+  for (int j = threadIdx.x; j < bins(0); j += kThreads)
+    if (s_h[j]) atomicAdd(hc + j, s_h[j]);
 }
 
 // ---- K1b': the streaming pass with 1-D TMA bulk copies -------------------------------------
@@ -339,7 +352,9 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
                                                               uint2* __restrict__ tile_info,
                                                               uint32_t* __restrict__ cand_idx,
                                                               float* __restrict__ cand_val, uint32_t cap,
-                                                              int vbf16) {
+                                                              int vbf16, uint32_t* __restrict__ hc) {
+  __shared__ uint32_t s_h[bins(0)];               // first-digit histogram of this CTA's candidates
+  for (int j = threadIdx.x; j < bins(0); j += kThreads) s_h[j] = 0;
   constexpr uint32_t kGB = kTile * (BF16 ? 2 : 4), kRB = kTile * 4, kSB = kGB + kRB;
   extern __shared__ __align__(128) uint8_t s_tiles[];          // kStages x {g tile, r tile}
   __shared__ __align__(8) uint64_t s_bar[kStages];
@@ -404,6 +419,13 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
       for (int e = 0; e < 4; ++e)
         if (tile < full_tiles || i + e < n) flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
     }
+    if (flags) {                                   // the select's first digit, for free
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          if ((flags >> (c * 4 + e)) & 1u) atomicAdd(&s_h[mag_key(a[c][e]) >> shift(0)], 1u);
+    }
     // Order-preserving compaction: one block scan of 4 x 16-bit per-vector counts.
     uint64_t packed = 0;
 #pragma unroll
@@ -440,6 +462,9 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
     tile_tail(a, flags, total, vec_base, excl, s_base[par], cap, base, n, tile < full_tiles, vbf16, r,
               cand_idx, cand_val);
   }
+  __syncthreads();
+  for (int j = threadIdx.x; j < bins(0); j += kThreads)
+    if (s_h[j]) atomicAdd(hc + j, s_h[j]);
 }
 
 // ---- K1c: exact radix select over the candidates (or the full array) ------------------------
@@ -449,9 +474,10 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
 template <int PASS>
 __device__ __forceinline__ void select_pass(const float* __restrict__ src, uint64_t N, uint32_t* sh,
                                             uint32_t* hist, uint32_t& prefix, uint64_t& need,
-                                            uint64_t* s_scan, cg::grid_group& grid) {
+                                            uint64_t* s_scan, cg::grid_group& grid, bool count = true) {
   constexpr int NB = bins(PASS);
   constexpr int SH = shift(PASS);
+  if (count) {
   for (int b = threadIdx.x; b < NB; b += kThreads) sh[b] = 0;
   __syncthreads();
   // Warp-aggregated increments: the candidates' keys crowd into few bins, so lanes with the same
@@ -473,6 +499,7 @@ __device__ __forceinline__ void select_pass(const float* __restrict__ src, uint6
   for (int b = threadIdx.x; b < NB; b += kThreads)
     if (sh[b]) atomicAdd(hist + b, sh[b]);
   grid.sync();
+  }
   uint64_t above;
   const int d = find_bin_desc<NB>(hist, need, &above, s_scan);
   need -= above;
@@ -529,7 +556,7 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
                                                           const uint32_t* __restrict__ cand_idx,
                                                           const uint2* __restrict__ tile_info,
                                                           uint32_t num_tiles, uint32_t cap, uint32_t* h0,
-                                                          uint32_t* h1, uint32_t* h2,
+                                                          uint32_t* h1, uint32_t* h2, uint32_t* hc,
                                                           uint64_t* tloc, uint64_t* boff, uint8_t* pairs) {
   cg::grid_group grid = cg::this_grid();
   __shared__ uint32_t sh[bins(0)];
@@ -551,7 +578,8 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
   }
   uint32_t prefix = 0;
   uint64_t need = k;
-  select_pass<0>(src, N, sh, h0, prefix, need, s_scan, grid);
+  // candidate mode: the stream pass already histogrammed the candidates' first digit (hc)
+  select_pass<0>(src, N, sh, mode ? h0 : hc, prefix, need, s_scan, grid, mode != 0);
   select_pass<1>(src, N, sh, h1, prefix, need, s_scan, grid);
   select_pass<2>(src, N, sh, h2, prefix, need, s_scan, grid);
   const uint32_t K = prefix;
@@ -747,6 +775,7 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   float* cval = reinterpret_cast<float*>(w + L.cand_val);
   const bool bf = gdt == LOWDIFF_BF16;
   const int vbf = vdt == LOWDIFF_BF16 ? 1 : 0;
+  uint32_t* hcand = reinterpret_cast<uint32_t*>(w + L.hc);
   static int use_tma = -1;
   if (use_tma < 0) {
     const char* e = getenv("LOWDIFF_STREAM_TMA");
@@ -758,19 +787,19 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
     const int smem = stream_tma_smem(bf);
     if (bf)
       LD_LAUNCH("compress_stream", s, stream_tma_kernel<true>, grid, kThreads, smem, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand);
     else
       LD_LAUNCH("compress_stream", s, stream_tma_kernel<false>, grid, kThreads, smem, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand);
   } else {
     int grid = stream_blocks(bf);
     if ((uint32_t)grid > L.num_tiles) grid = (int)L.num_tiles;
     if (bf)
       LD_LAUNCH("compress_stream", s, stream_kernel<true>, grid, kThreads, 0, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand);
     else
       LD_LAUNCH("compress_stream", s, stream_kernel<false>, grid, kThreads, 0, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand);
   }
 
   {
@@ -805,7 +834,7 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
     uint32_t cap = L.cap, nt = L.num_tiles;
     void* args[] = {(void*)&rr, (void*)&n, (void*)&k, (void*)&ctl, (void*)&cval, (void*)&cidx_c,
                     (void*)&tiles_c, (void*)&nt, (void*)&cap, (void*)&h0, (void*)&h1, (void*)&h2,
-                    (void*)&tloc, (void*)&boff, (void*)&pp};
+                    (void*)&hcand, (void*)&tloc, (void*)&boff, (void*)&pp};
     ProfScope prof("compress_select", s);
     const void* fn = vdt == LOWDIFF_BF16 ? (const void*)select_kernel<true> : (const void*)select_kernel<false>;
     LD_CUDA(cudaLaunchCooperativeKernel(fn, sel_grid, kThreads, args, 0, s), "select launch");
