@@ -92,7 +92,7 @@ class LowDiffLoop:
             self.full_pool = [{k: torch.empty(L, dtype=torch.float32, pin_memory=True) for k in keys}
                               for _ in range(retain_fulls + 1)]
             self.pool = [torch.empty(self.rec_cap, dtype=torch.uint8, pin_memory=True)
-                         for _ in range(retain_fulls * (full_every // B) + 2)]
+                         for _ in range(min(retain_fulls * (full_every // B) + 2, 16))]   # more on demand
 
     # ---- one training iteration ---------------------------------------------------------------
     def step(self, grad: torch.Tensor):
