@@ -239,6 +239,30 @@ lowdiff_status lowdiff_update(lowdiff_state* st, const lowdiff_opt* opt, const l
                               void* ws, uint64_t ws_bytes, lowdiff_stream_t stream);
 
 /* ---------------------------------------------------------------------------------------------
+ * (6) LowDiff+ — training without gradient compression (§5, Algorithm 2; SURVEY
+ *     §8(f) NEXT-4). The dense synchronized gradient G_t of the shard [lo, hi) updates
+ *       lowdiff_dense_update: the GPU model in place, "M^G_{t+1} <- M^G_t + Adam(o_t, G_t)"
+ *                             (Alg. 2 line 7), asynchronously on `stream`;
+ *       lowdiff_host_update:  the CPU-resident replica in place, "M^C_{t+1} <- M^C_t + Adam(o_t,
+ *                             G_t)" (line 12; the in-memory checkpoint), synchronously
+ *                             on the calling thread plus `threads` - 1 workers (>= 1).
+ *     Both run the same IEEE fp32 op sequence as lowdiff_replay / lowdiff_update (SGD with
+ *     optional weight decay, SGD-momentum, Adam; readings #16, #18, #19), so after the
+ *     same gradients the replica equals the GPU model bit for bit ("keep it synchronized").
+ *   st: x (and m, v as the optimizer needs) over [lo, hi): DEVICE pointers for the GPU update,
+ *       HOST pointers for the host update; x0/m0/v0/x_bf16 must be NULL (in place only);
+ *       st->t, st->adam_step, st->momentum_initialized advance by one step.
+ *   grad: hi - lo gradient values, fp32 or bf16 (gdt), device (16-byte aligned) resp. host.
+ *   lr: this iteration's learning rate.
+ * Errors: EINVAL (null/misaligned pointers, bad dtype, x0/m0/v0/x_bf16 set), EUNSUPPORTED (Adam
+ *   with weight decay), ECUDA.
+ * ------------------------------------------------------------------------------------------- */
+lowdiff_status lowdiff_dense_update(lowdiff_state* st, const lowdiff_opt* opt, const void* grad,
+                                    lowdiff_dtype gdt, float lr, lowdiff_stream_t stream);
+lowdiff_status lowdiff_host_update(lowdiff_state* st, const lowdiff_opt* opt, const void* grad,
+                                   lowdiff_dtype gdt, float lr, int32_t threads);
+
+/* ---------------------------------------------------------------------------------------------
  * (5b) Parallel recovery — §4.4 "Parallel recovery module" on Eq. 2 (P:92,
  *     M_n = C^F + C^D_1 + ... + C^D_n): for plain SGD (weight_decay 0) over SUM records that share
  *     one constant lr, the chain's differentials are first merged among themselves — ONE multiway

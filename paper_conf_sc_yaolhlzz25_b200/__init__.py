@@ -79,7 +79,7 @@ EXPORTS = [
     "lowdiff_profile_enable", "lowdiff_profile_query", "lowdiff_compress_stats",
     "lowdiff_debug_force_threshold", "lowdiff_wasted_time", "lowdiff_optimal_config",
     "lowdiff_replay_parallel_workspace_size", "lowdiff_replay_parallel",
-    "lowdiff_update_workspace_size", "lowdiff_update",
+    "lowdiff_update_workspace_size", "lowdiff_update", "lowdiff_dense_update", "lowdiff_host_update",
 ]
 
 _lib = None
@@ -133,6 +133,8 @@ def lib() -> C.CDLL:
         "lowdiff_optimal_config": ([vp, vp, vp, vp, vp], i32),
         "lowdiff_update_workspace_size": ([vp, vp], i32),
         "lowdiff_update": ([vp, vp, vp, vp, u64, vp], i32),
+        "lowdiff_dense_update": ([vp, vp, vp, i32, C.c_float, vp], i32),
+        "lowdiff_host_update": ([vp, vp, vp, i32, C.c_float, i32], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -489,6 +491,49 @@ def update(state: dict, opt: dict, g_t, ws=None, stream=None) -> dict:
         ws = workspace(b.value, state["x"].device, "update")
     _check(lib().lowdiff_update(C.byref(st), C.byref(o), C.byref(view), _cuda(ws, "ws"), ws.numel(),
                                 _stream(stream)), "update")
+    state["t"], state["adam_step"] = st.t, st.adam_step
+    state["momentum_initialized"] = st.momentum_initialized
+    return state
+
+
+def _dense_args(state: dict, opt: dict, grad: torch.Tensor, device: bool):
+    o = Opt(_KIND[opt["kind"]], opt.get("momentum", 0.0), opt.get("dampening", 0.0),
+            opt.get("weight_decay", 0.0), opt.get("beta1", 0.9), opt.get("beta2", 0.999),
+            opt.get("eps", 1e-8), int(opt.get("nesterov", 0)), 0)
+    if grad.dtype not in (torch.float32, torch.bfloat16) or not grad.is_contiguous():
+        raise ValueError("grad must be a contiguous fp32/bf16 tensor")
+    L = state["hi"] - state["lo"]
+    for key in ("x", "m", "v"):
+        t = state.get(key)
+        if t is not None and (t.is_cuda != device or t.dtype != torch.float32 or t.numel() != L
+                              or not t.is_contiguous()):
+            raise ValueError(f"state[{key!r}] must be a contiguous fp32 {'CUDA' if device else 'CPU'} tensor of {L}")
+    if grad.is_cuda != device or grad.numel() != L:
+        raise ValueError(f"grad must be a {'CUDA' if device else 'CPU'} tensor of {L} values")
+    ptr = lambda key: state[key].data_ptr() if state.get(key) is not None else None
+    st = State(ptr("x"), ptr("m"), ptr("v"), None, state["n"], state["lo"], state["hi"], state["t"],
+               state["adam_step"], state["momentum_initialized"], None, None, None)
+    return o, st, BF16 if grad.dtype == torch.bfloat16 else F32
+
+
+def dense_update(state: dict, opt: dict, grad: torch.Tensor, lr: float, stream=None) -> dict:
+    """LowDiff+ GPU model update (Alg. 2 line 7): one dense optimizer step of the shard state from
+    the dense gradient (CUDA fp32/bf16), in place, asynchronous on the stream."""
+    o, st, gdt = _dense_args(state, opt, grad, True)
+    _check(lib().lowdiff_dense_update(C.byref(st), C.byref(o), grad.data_ptr(), gdt, float(lr), _stream(stream)),
+           "dense_update")
+    state["t"], state["adam_step"] = st.t, st.adam_step
+    state["momentum_initialized"] = st.momentum_initialized
+    return state
+
+
+def host_update(state: dict, opt: dict, grad: torch.Tensor, lr: float, threads: int = 0) -> dict:
+    """LowDiff+ CPU replica update (Alg. 2 line 12): the same step on host tensors, `threads`
+    workers (0 = all cores). Blocks the calling thread (ctypes releases the GIL meanwhile)."""
+    o, st, gdt = _dense_args(state, opt, grad, False)
+    threads = threads or os.cpu_count() or 1
+    _check(lib().lowdiff_host_update(C.byref(st), C.byref(o), grad.data_ptr(), gdt, float(lr), int(threads)),
+           "host_update")
     state["t"], state["adam_step"] = st.t, st.adam_step
     state["momentum_initialized"] = st.momentum_initialized
     return state

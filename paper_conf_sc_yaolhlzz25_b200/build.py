@@ -36,7 +36,12 @@ def nccl_dir() -> str:
 
 
 def sources() -> list[str]:
-    return sorted(glob.glob(os.path.join(CSRC, "*.cu")))
+    return sorted(glob.glob(os.path.join(CSRC, "*.cu"))) + sorted(glob.glob(os.path.join(CSRC, "*.cpp")))
+
+
+# plain C++ (the LowDiff+ host replica update): IEEE fp32 with no FMA contraction, vectorised
+CXX = os.environ.get("CXX", "g++")
+CXXFLAGS = ["-O3", "-std=c++17", "-fPIC", "-pthread", "-ffp-contract=off", "-fno-math-errno", "-g"]
 
 
 def _deps() -> list[str]:
@@ -61,12 +66,15 @@ def build(force: bool = False, verbose: bool = False) -> str:
     def compile_one(src: str) -> str:
         obj = os.path.join(BUILD, os.path.basename(src) + ".o")
         extra = os.environ.get("LOWDIFF_NVCC_EXTRA", "").split()   # experiments, e.g. -DLOWDIFF_REPLAY_MINB=4
-        cmd = [NVCC, *ARCH, *CFLAGS, *extra, *inc, "-c", src, "-o", obj]
+        if src.endswith(".cpp"):
+            cmd = [CXX, *CXXFLAGS, "-I", INCLUDE, "-I", CSRC, "-c", src, "-o", obj]
+        else:
+            cmd = [NVCC, *ARCH, *CFLAGS, *extra, *inc, "-c", src, "-o", obj]
         if verbose:
             print(" ".join(cmd), flush=True)
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
-            raise RuntimeError(f"nvcc failed for {src}:\n{r.stdout}\n{r.stderr}")
+            raise RuntimeError(f"compile failed for {src}:\n{r.stdout}\n{r.stderr}")
         if verbose and r.stderr.strip():
             print(r.stderr, file=sys.stderr)
         return obj
@@ -76,7 +84,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     lib = os.path.join(nd, "lib")
     tmp = SO + f".tmp{os.getpid()}"
     cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-L", lib, "-l:libnccl.so.2",
-           "-Xlinker", f"-rpath,{lib}", "-cudart", "static"]
+           "-Xlinker", f"-rpath,{lib}", "-cudart", "static", "-lpthread"]
     if verbose:
         print(" ".join(cmd), flush=True)
     r = subprocess.run(cmd, capture_output=True, text=True)

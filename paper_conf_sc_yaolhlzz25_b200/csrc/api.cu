@@ -470,6 +470,34 @@ lowdiff_status lowdiff_update(lowdiff_state* st, const lowdiff_opt* opt, const l
   return replay_run(st, opt, &r, 1, ws, (cudaStream_t)stream);
 }
 
+static lowdiff_status check_dense(const lowdiff_state* st, const lowdiff_opt* opt, const void* grad, int gdt) {
+  lowdiff_status s = check_state(st, opt);
+  if (s) return s;
+  if (!grad) return fail(LOWDIFF_EINVAL, "dense update: null gradient");
+  if (gdt != LOWDIFF_F32 && gdt != LOWDIFF_BF16) return fail(LOWDIFF_EINVAL, "dense update: gradient dtype");
+  if (st->x0 || st->m0 || st->v0 || st->x_bf16)
+    return fail(LOWDIFF_EINVAL, "dense update: in place only (x0/m0/v0/x_bf16 must be NULL)");
+  return LOWDIFF_OK;
+}
+
+lowdiff_status lowdiff_dense_update(lowdiff_state* st, const lowdiff_opt* opt, const void* grad, lowdiff_dtype gdt,
+                                    float lr, lowdiff_stream_t stream) {
+  lowdiff_status s = check_dense(st, opt, grad, gdt);
+  if (s) return s;
+  if (!aligned16(grad)) return fail(LOWDIFF_EINVAL, "dense_update: misaligned gradient");
+  return dense_update_run(st, opt, grad, gdt, lr, (cudaStream_t)stream);
+}
+
+lowdiff_status lowdiff_host_update(lowdiff_state* st, const lowdiff_opt* opt, const void* grad, lowdiff_dtype gdt,
+                                   float lr, int32_t threads) {
+  lowdiff_status s = check_dense(st, opt, grad, gdt);
+  if (s) return s;
+  DenseStep d;
+  dense_update_scalars(st, opt, lr, &d);
+  host_update_run(d, st->x, st->m, st->v, grad, gdt == LOWDIFF_BF16, st->hi - st->lo, threads);
+  return LOWDIFF_OK;
+}
+
 static lowdiff_status parallel_supported(const lowdiff_opt* o, const std::vector<RecInfo>& R) {
   if (o->kind != LOWDIFF_OPT_SGD || o->weight_decay != 0.0)
     return fail(LOWDIFF_EUNSUPPORTED, "replay_parallel: plain SGD (weight_decay 0) only");

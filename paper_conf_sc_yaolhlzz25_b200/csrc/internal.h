@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include "dense_step.h"
 #include "lowdiff.h"
 
 namespace lowdiff {
@@ -85,5 +86,10 @@ lowdiff_status replay_run(lowdiff_state* st, const lowdiff_opt* o, const RecInfo
 uint64_t replay_parallel_ws_bytes(uint32_t nrec, uint64_t entries, uint64_t lo, uint64_t hi);
 lowdiff_status replay_parallel_run(lowdiff_state* st, const RecInfo* recs, uint32_t nrec, void* ws,
                                    cudaStream_t s);
+
+// ---- LowDiff+ dense updates (plus.cu, host_update.cpp) ----------------------------------------
+void dense_update_scalars(lowdiff_state* st, const lowdiff_opt* o, float lr, DenseStep* d);
+lowdiff_status dense_update_run(lowdiff_state* st, const lowdiff_opt* o, const void* grad, int gdt, float lr,
+                                cudaStream_t s);
 
 }  // namespace lowdiff
