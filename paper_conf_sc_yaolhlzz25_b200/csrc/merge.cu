@@ -90,7 +90,7 @@ __device__ __forceinline__ float list_val(const ListSet& ls, int l, uint64_t e) 
 // items[i] = (first fine window, number of fine windows).
 __global__ void __launch_bounds__(kPlanThreads) plan_kernel(int L, const uint32_t* __restrict__ starts,
                                                             uint32_t num_w, uint32_t G, uint32_t sparse_max,
-                                                            MCtl* ctl, uint2* __restrict__ items) {
+                                                            int keep_groups, MCtl* ctl, uint2* __restrict__ items) {
   __shared__ uint32_t s_warp[kPlanThreads / 32];
   __shared__ uint32_t s_carry;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -119,7 +119,8 @@ __global__ void __launch_bounds__(kPlanThreads) plan_kernel(int L, const uint32_
         const uint32_t* st = starts + (uint64_t)l * (num_w + 1);
         e += st[fe] - st[fs];
       }
-      cnt = (e <= (uint64_t)sparse_max || fe - fs == 1) ? 1u : fe - fs;
+      // keep_groups: bitmap-sized groups stay whole (the bitmap path takes any entry count)
+      cnt = (keep_groups || e <= (uint64_t)sparse_max || fe - fs == 1) ? 1u : fe - fs;
     }
     uint32_t incl = cnt;
 #pragma unroll
@@ -153,9 +154,19 @@ struct DenseSmem {
 struct SparseSmem {
   uint64_t sk[2][kCap];          // (idx - w0) << 40 | list << 32 | load position; merge ping-pong
 };
+constexpr int kBmLists = 32;                // lists the bitmap path handles
+constexpr int kWords = kW / 32;             // bitmap words per fine window
+constexpr int kBmWords = 6144;              // list x word capacity of a bitmap item (24 KB)
+constexpr int kBmMaxWords = 768;            // words (6 windows) per bitmap item
+struct BitmapSmem {
+  uint32_t bm[kBmWords];           // per list, the item's occupied slots (list-major)
+  uint64_t wpre[kBmMaxWords];      // per word: (# unique slots before it) << 32 | # entries before it
+  uint32_t orw[kBmMaxWords];       // per word: slots occupied by any list
+};
 union ItemSmem {
   DenseSmem d;
   SparseSmem s;
+  BitmapSmem b;
 };
 
 template <int KIND, bool BF16>
@@ -166,7 +177,8 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
                                                          uint32_t* __restrict__ stg_idx,
                                                          uint32_t* __restrict__ stg_val,
                                                          uint8_t* __restrict__ out_it,
-                                                         float* __restrict__ out_ent, uint32_t sparse_max) {
+                                                         float* __restrict__ out_ent, uint32_t sparse_max,
+                                                         uint32_t bitmap_min) {
   __shared__ ItemSmem sm;
   __shared__ uint32_t s_beg[kMaxLists], s_len[kMaxLists], s_off[kMaxLists + 1];
   __shared__ uint64_t s_scan[kThreads / 32];
@@ -203,7 +215,77 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
     const uint32_t E = (uint32_t)tot_e;
     const uint32_t e0 = s_e0;
     uint64_t tot;
-    if (E <= sparse_max) {
+    auto list_of = [&](uint32_t x) -> int {        // list l with s_off[l] <= x < s_off[l+1]
+      int a = 0, b = L - 1;
+      while (a < b) {
+        const int mid = (a + b + 1) >> 1;
+        if (s_off[mid] <= x) a = mid; else b = mid - 1;
+      }
+      return a;
+    };
+    const uint32_t NW = it.y * kWords;            // bitmap words of this item
+    const bool bm_shape = KIND == kMergeStack && L <= kBmLists && (uint32_t)L * NW <= (uint32_t)kBmWords &&
+                          NW <= (uint32_t)kBmMaxWords;
+    if (bm_shape && (E >= bitmap_min * it.y || (E > sparse_max && it.y > 1))) {
+      // ---- bitmap item (STACK, dense enough): per list a bitmap of the item's occupied slots;
+      //      per word the (unique, entry) counts and their exclusive scan; then every entry finds
+      //      its final position with popcounts alone:
+      //        pos = e0 + entries in earlier words + entries of this word at lower slots
+      //              + lists before its own with the same slot (iteration order)
+      //      and the first entry of a slot (rank 0) writes the unique head. No sorting.
+      for (uint32_t j = tid; j < (uint32_t)L * NW; j += kThreads) sm.b.bm[j] = 0;
+      __syncthreads();
+      for (uint32_t x = tid; x < E; x += kThreads) {
+        const int a = list_of(x);
+        const uint32_t slot = ls.list[a].idx[s_beg[a] + (x - s_off[a])] - (uint32_t)w0;
+        atomicOr(&sm.b.bm[a * NW + (slot >> 5)], 1u << (slot & 31));
+      }
+      __syncthreads();
+      // each thread owns q consecutive words: their counts, a block scan, then the per-word prefix
+      const uint32_t q = (NW + kThreads - 1) / kThreads, w_a = tid * q, w_e = min(NW, w_a + q);
+      uint64_t mine = 0;
+      for (uint32_t wd = w_a; wd < w_e; ++wd) {
+        uint32_t orv = 0, c = 0;
+        for (int l = 0; l < L; ++l) {
+          const uint32_t bw = sm.b.bm[l * NW + wd];
+          orv |= bw;
+          c += __popc(bw);
+        }
+        sm.b.orw[wd] = orv;
+        mine += ((uint64_t)__popc(orv) << 32) | c;
+      }
+      uint64_t run = block_exclusive_scan(mine, s_scan, &tot);
+      for (uint32_t wd = w_a; wd < w_e; ++wd) {
+        sm.b.wpre[wd] = run;
+        uint32_t c = 0;
+        for (int l = 0; l < L; ++l) c += __popc(sm.b.bm[l * NW + wd]);
+        run += ((uint64_t)__popc(sm.b.orw[wd]) << 32) | c;
+      }
+      __syncthreads();
+      for (uint32_t x = tid; x < E; x += kThreads) {
+        const int a = list_of(x);
+        const uint64_t e = s_beg[a] + (x - s_off[a]);
+        const uint32_t slot = ls.list[a].idx[e] - (uint32_t)w0;
+        const uint32_t wd = slot >> 5, bit = 1u << (slot & 31), below = bit - 1u;
+        uint32_t cb = 0, rank = 0;
+        for (int l = 0; l < L; ++l) {
+          const uint32_t bw = sm.b.bm[l * NW + wd];
+          cb += __popc(bw & below);
+          rank += (l < a && (bw & bit)) ? 1u : 0u;
+        }
+        const uint64_t pw = sm.b.wpre[wd];
+        const uint32_t pos = e0 + (uint32_t)pw + cb + rank;
+        out_it[pos] = (uint8_t)a;
+        out_ent[pos] = list_val<BF16>(ls, a, e);
+        if (rank == 0) {
+          const uint32_t u = e0 + (uint32_t)(pw >> 32) + __popc(sm.b.orw[wd] & below);
+          stg_idx[u] = (uint32_t)(w0 + slot);
+          stg_val[u] = pos;                        // off[] = the head's entry position
+        }
+      }
+      tot >>= 32;                                  // unique slots of the item
+      dense_clean = false;                         // the bitmap arrays alias cnt[]
+    } else if (E <= sparse_max) {
       // ---- sparse item: load the lists' segments (each sorted by index) as runs of unique
       //      composite keys (index, list), then merge runs pairwise, ceil(log2 L) rounds: a key's
       //      rank in the merged run = its rank in its own run + the number of smaller keys in the
@@ -620,7 +702,21 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
   uint32_t sparse_max = kCap;       // items with more entries take the dense (one window) path
   if (const char* e = getenv("LOWDIFF_MERGE_SPARSE_MAX")) sparse_max = (uint32_t)atoi(e);
   if (sparse_max > (uint32_t)kCap) sparse_max = kCap;
-  LD_LAUNCH("merge_plan", s, plan_kernel, 1, kPlanThreads, 0, ls.L, starts, M.num_w, G, sparse_max, ctl,
+  // STACK merges of dense-enough differentials: one window per item through the bitmap path
+  uint32_t bitmap_min = 96;         // entries per window from which the bitmap path is used
+  if (const char* e = getenv("LOWDIFF_MERGE_BITMAP_MIN")) bitmap_min = (uint32_t)atoi(e);
+  // (measured: with 32 lists the popcount work per entry grows past the sparse run merging, so
+  // the bitmap path is used up to 16 lists; groups stay small enough to leave >= 4 items per CTA)
+  int keep_groups = 0;
+  const uint32_t merge_ctas = 6u * kNumSMs;
+  if (kind == kMergeStack && ls.L <= 16 && per_w >= (double)bitmap_min) {
+    G = 1;                          // groups of bitmap size: as many windows as fit (power of 2)
+    while (2 * G * kWords <= (uint32_t)kBmMaxWords && (uint32_t)ls.L * 2 * G * kWords <= (uint32_t)kBmWords &&
+           M.num_w / (2 * G) >= 4 * merge_ctas)
+      G <<= 1;
+    keep_groups = 1;
+  }
+  LD_LAUNCH("merge_plan", s, plan_kernel, 1, kPlanThreads, 0, ls.L, starts, M.num_w, G, sparse_max, keep_groups, ctl,
             items);
 
   const int grid = (int)(M.num_w < 6u * kNumSMs ? M.num_w : 6u * kNumSMs);   // 6 CTAs/SM (37 KB smem)
@@ -634,16 +730,16 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
   const char* cls = record ? "merge" : "coalesce";
   if (kind == kCoalesce && ls.bf16)
     LD_LAUNCH(cls, s, (merge_kernel<kCoalesce, true>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
-              ucnt, epre, sidx, sval, oit, oent, sparse_max);
+              ucnt, epre, sidx, sval, oit, oent, sparse_max, bitmap_min);
   else if (kind == kCoalesce)
     LD_LAUNCH(cls, s, (merge_kernel<kCoalesce, false>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
-              ucnt, epre, sidx, sval, oit, oent, sparse_max);
+              ucnt, epre, sidx, sval, oit, oent, sparse_max, bitmap_min);
   else if (kind == kMergeSum)
     LD_LAUNCH(cls, s, (merge_kernel<kMergeSum, false>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
-              ucnt, epre, sidx, sval, oit, oent, sparse_max);
+              ucnt, epre, sidx, sval, oit, oent, sparse_max, bitmap_min);
   else
     LD_LAUNCH(cls, s, (merge_kernel<kMergeStack, false>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
-              ucnt, epre, sidx, sval, oit, oent, sparse_max);
+              ucnt, epre, sidx, sval, oit, oent, sparse_max, bitmap_min);
   LD_LAUNCH(cls, s, ucount_scan_kernel, 1, kPlanThreads, 0, ls, M.num_w, starts, ctl, ucnt, upre,
             kind == kCoalesce ? d_out_nnz : nullptr);
   uint32_t* didx = record ? reinterpret_cast<uint32_t*>(w + M.widx) : out_idx;
