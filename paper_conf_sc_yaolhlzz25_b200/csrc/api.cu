@@ -211,7 +211,8 @@ lowdiff_status lowdiff_coalesce(const void* gathered, int32_t nranks, uint64_t k
                                 lowdiff_stream_t stream) {
   lowdiff_status s = check_coalesce_args(nranks, k, vdt, lo, hi);
   if (s) return s;
-  if (!gathered || !out_idx || !out_val || !d_out_nnz || !ws || !aligned16(gathered) || !aligned16(ws))
+  if (!gathered || !out_idx || !out_val || !d_out_nnz || !ws || !aligned16(gathered) || !aligned16(ws) ||
+      !aligned16(out_idx) || !aligned16(out_val))
     return fail(LOWDIFF_EINVAL, "coalesce: null or misaligned pointer");
   const uint64_t need = (uint64_t)nranks * k < hi - lo ? (uint64_t)nranks * k : hi - lo;
   if (out_cap < need) return fail(LOWDIFF_EINVAL, "coalesce: out_cap %llu < min(P*k, hi-lo) = %llu",
@@ -252,7 +253,8 @@ lowdiff_status lowdiff_allgather_sparse(lowdiff_comm* comm, const void* pairs, u
   uint64_t need = 0;
   lowdiff_status s = lowdiff_allgather_sparse_workspace_size(P, k, vdt, lo, hi, &need);
   if (s) return s;
-  if (!pairs || !ws || !aligned16(pairs) || !aligned16(ws)) return fail(LOWDIFF_EINVAL, "allgather_sparse: pointer");
+  if (!pairs || !ws || !aligned16(pairs) || !aligned16(ws) || !aligned16(out_idx) || !aligned16(out_val))
+    return fail(LOWDIFF_EINVAL, "allgather_sparse: pointer");
   if (ws_bytes < need) return fail(LOWDIFF_EWORKSPACE, "allgather_sparse: workspace too small");
   uint64_t cws = 0;
   lowdiff_coalesce_workspace_size(P, k, vdt, lo, hi, &cws);

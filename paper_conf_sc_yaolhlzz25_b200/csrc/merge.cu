@@ -553,7 +553,27 @@ __global__ void __launch_bounds__(kThreads) single_list_kernel(const uint32_t* _
   }
   __syncthreads();
   const uint64_t first = s_first, cnt = s_last - s_first;
-  for (uint64_t e = (uint64_t)blockIdx.x * kThreads + threadIdx.x; e < cnt; e += (uint64_t)gridDim.x * kThreads) {
+  uint64_t done = 0;
+  if ((first & 3) == 0) {                          // aligned: 4 entries per thread, 128-bit idx I/O
+    const uint64_t c4 = cnt / 4;
+    for (uint64_t q = (uint64_t)blockIdx.x * kThreads + threadIdx.x; q < c4; q += (uint64_t)gridDim.x * kThreads) {
+      const uint64_t e = q * 4;
+      *reinterpret_cast<uint4*>(out_idx + e) = *reinterpret_cast<const uint4*>(idx + first + e);
+      float v[4];
+      if constexpr (BF16) {
+        const uint2 u = *reinterpret_cast<const uint2*>(static_cast<const uint16_t*>(val) + first + e);
+        v[0] = __uint_as_float(u.x << 16); v[1] = __uint_as_float(u.x & 0xFFFF0000u);
+        v[2] = __uint_as_float(u.y << 16); v[3] = __uint_as_float(u.y & 0xFFFF0000u);
+      } else {
+        const float4 t = *reinterpret_cast<const float4*>(static_cast<const float*>(val) + first + e);
+        v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
+      }
+      *reinterpret_cast<float4*>(out_val + e) =          // the definition's "/ P" with P = 1 (exact)
+          make_float4(__fdiv_rn(v[0], 1.0f), __fdiv_rn(v[1], 1.0f), __fdiv_rn(v[2], 1.0f), __fdiv_rn(v[3], 1.0f));
+    }
+    done = c4 * 4;
+  }
+  for (uint64_t e = done + (uint64_t)blockIdx.x * kThreads + threadIdx.x; e < cnt; e += (uint64_t)gridDim.x * kThreads) {
     out_idx[e] = idx[first + e];
     float v;
     if constexpr (BF16) v = __uint_as_float(((uint32_t) static_cast<const uint16_t*>(val)[first + e]) << 16);
@@ -669,7 +689,7 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
   (void)out_cap;
   const bool record = kind != kCoalesce;
   if (kind == kCoalesce && ls.L == 1) {
-    uint64_t g = (ls.list[0].len + kThreads - 1) / kThreads;
+    uint64_t g = (ls.list[0].len / 4 + kThreads - 1) / kThreads;
     if (g > 4ull * kNumSMs) g = 4ull * kNumSMs;
     if (g < 1) g = 1;
     if (ls.bf16)
