@@ -484,15 +484,26 @@ __device__ __forceinline__ void select_pass(const float* __restrict__ src, uint6
   // bin are combined (__match_any_sync) into one shared-memory atomic.
   const int lane = threadIdx.x & 31;
   const uint64_t stride = (uint64_t)gridDim.x * kThreads;
-  for (uint64_t base = (uint64_t)blockIdx.x * kThreads + (threadIdx.x & ~31u); base < N; base += stride) {
-    const uint64_t i = base + lane;
-    const uint32_t key = i < N ? mag_key(src[i]) : 0u;
-    const bool take = i < N && (PASS == 0 || (key >> shift(PASS > 0 ? PASS - 1 : 0)) == prefix);
-    const uint32_t act = __ballot_sync(0xFFFFFFFFu, take);
-    if (take) {
-      const uint32_t bin = (key >> SH) & (NB - 1);
-      const uint32_t peers = __match_any_sync(act, bin);
-      if (lane == __ffs(peers) - 1) atomicAdd(&sh[bin], (uint32_t)__popc(peers));
+  constexpr int U = 4;                             // loads in flight per thread
+  for (uint64_t base = (uint64_t)blockIdx.x * kThreads + (threadIdx.x & ~31u); base < N; base += U * stride) {
+    uint32_t keys[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint64_t i = base + u * stride + lane;
+      keys[u] = i < N ? mag_key(src[i]) : 0u;
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if (base + u * stride >= N) break;           // warp-uniform
+      const uint64_t i = base + u * stride + lane;
+      const uint32_t key = keys[u];
+      const bool take = i < N && (PASS == 0 || (key >> shift(PASS > 0 ? PASS - 1 : 0)) == prefix);
+      const uint32_t act = __ballot_sync(0xFFFFFFFFu, take);
+      if (take) {
+        const uint32_t bin = (key >> SH) & (NB - 1);
+        const uint32_t peers = __match_any_sync(act, bin);
+        if (lane == __ffs(peers) - 1) atomicAdd(&sh[bin], (uint32_t)__popc(peers));
+      }
     }
   }
   __syncthreads();
@@ -619,6 +630,7 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
     const uint64_t t = tw + (lane >> glog);
     const uint2 ti = t < num_tiles ? segment(t) : make_uint2(0u, 0u);
     uint32_t gt = 0, eq = 0;
+#pragma unroll 4
     for (uint32_t j = gl; j < ti.y; j += g) {
       const uint32_t key = mag_key(vsrc[(uint64_t)ti.x + j]);
       gt += key > K;
@@ -650,44 +662,66 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
     if (vp + threadIdx.x < ve) pairs[vp + threadIdx.x] = 0;
   }
   const uint32_t lt = (1u << gl) - 1;
-  for (uint64_t tw = tfirst - (lane >> glog); tw < num_tiles; tw += wstride) {   // warp-uniform
+  // the next round's tile (segment, prefix) is loaded while the current one is emitted, and the
+  // group's loads of two iterations are issued together: the loop is load-latency bound
+  auto tinfo = [&](uint64_t tw, uint2& ti, uint64_t& tp) {
     const uint64_t t = tw + (lane >> glog);
     const bool tv = t < num_tiles;
-    const uint2 ti = tv ? segment(t) : make_uint2(0u, 0u);
-    const uint64_t tp = tv ? tcnt[t] + __ldcg(boff + G + (t >> ts_log)) : 0;
+    ti = tv ? segment(t) : make_uint2(0u, 0u);
+    tp = tv ? tcnt[t] + __ldcg(boff + G + (t >> ts_log)) : 0;
+  };
+  uint64_t tw = tfirst - (lane >> glog);
+  uint2 ti = make_uint2(0u, 0u);
+  uint64_t tp = 0;
+  if (tw < num_tiles) tinfo(tw, ti, tp);
+  for (; tw < num_tiles; tw += wstride) {          // warp-uniform
+    uint2 nti = make_uint2(0u, 0u);
+    uint64_t ntp = 0;
+    if (tw + wstride < num_tiles) tinfo(tw + wstride, nti, ntp);
     uint64_t gtb = tp >> 32, eqb = tp & 0xFFFFFFFFull;
     const uint32_t len_max = __reduce_max_sync(0xFFFFFFFFu, ti.y);
-    for (uint32_t j0 = 0; j0 < len_max; j0 += g) {
-      const uint32_t j = j0 + gl;
-      const bool in = j < ti.y;
-      float a = 0.f;
-      uint32_t idx = 0;
-      if (in) {
-        a = vsrc[(uint64_t)ti.x + j];
-        idx = mode ? ti.x + j : cand_idx[(uint64_t)ti.x + j];
+    for (uint32_t j0 = 0; j0 < len_max; j0 += 2 * g) {
+      float a2[2];
+      uint32_t id2[2];
+      bool in2[2];
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const uint32_t j = j0 + h * g + gl;
+        in2[h] = j < ti.y;
+        a2[h] = in2[h] ? vsrc[(uint64_t)ti.x + j] : 0.f;
+        id2[h] = in2[h] ? (mode ? ti.x + j : cand_idx[(uint64_t)ti.x + j]) : 0u;
       }
-      const uint32_t key = mag_key(a);
-      const bool isg = in && key > K, ise = in && key == K;
-      const uint32_t bg = (__ballot_sync(0xFFFFFFFFu, isg) >> gshift) & gmask;
-      const uint32_t be = (__ballot_sync(0xFFFFFFFFu, ise) >> gshift) & gmask;
-      const uint64_t myeq = eqb + __popc(be & lt);
-      if (isg || (ise && myeq < m)) {
-        const uint64_t pos = gtb + __popc(bg & lt) + (myeq < m ? myeq : m);
-        out_idx[pos] = idx;
-        if constexpr (VBF16) {
-          const __nv_bfloat16 h = __float2bfloat16_rn(a);
-          reinterpret_cast<__nv_bfloat16*>(out_val)[pos] = h;
-          if (mode) r[idx] = a - __bfloat162float(h);   // exact (Sterbenz), reading #8
-        } else {
-          reinterpret_cast<float*>(out_val)[pos] = a;
-          if (mode) r[idx] = 0.0f;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        if (j0 + h * g >= len_max) break;          // warp-uniform
+        const float a = a2[h];
+        const uint32_t idx = id2[h];
+        const bool in = in2[h];
+        const uint32_t key = mag_key(a);
+        const bool isg = in && key > K, ise = in && key == K;
+        const uint32_t bg = (__ballot_sync(0xFFFFFFFFu, isg) >> gshift) & gmask;
+        const uint32_t be = (__ballot_sync(0xFFFFFFFFu, ise) >> gshift) & gmask;
+        const uint64_t myeq = eqb + __popc(be & lt);
+        if (isg || (ise && myeq < m)) {
+          const uint64_t pos = gtb + __popc(bg & lt) + (myeq < m ? myeq : m);
+          out_idx[pos] = idx;
+          if constexpr (VBF16) {
+            const __nv_bfloat16 hb = __float2bfloat16_rn(a);
+            reinterpret_cast<__nv_bfloat16*>(out_val)[pos] = hb;
+            if (mode) r[idx] = a - __bfloat162float(hb);   // exact (Sterbenz), reading #8
+          } else {
+            reinterpret_cast<float*>(out_val)[pos] = a;
+            if (mode) r[idx] = 0.0f;
+          }
+        } else if (in && !mode) {
+          r[idx] = a;                              // a rejected candidate keeps all of a
         }
-      } else if (in && !mode) {
-        r[idx] = a;                                // a rejected candidate keeps all of a
+        gtb += __popc(bg);
+        eqb += __popc(be);
       }
-      gtb += __popc(bg);
-      eqb += __popc(be);
     }
+    ti = nti;
+    tp = ntp;
   }
 }
 
