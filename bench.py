@@ -47,6 +47,9 @@ def parse_args():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-graph", action="store_true", help="time eager launches (no CUDA graph)")
+    ap.add_argument("--sync", default="p2p", choices=["p2p", "nccl"],
+                    help="N > 1: all-gather fused with the coalesce over peer memory (p2p, default) or "
+                         "ncclAllGather + coalesce (nccl)")
     ap.add_argument("--grad-pool", type=int, default=0,
                     help="distinct resident gradients cycled through (0 = one per iteration of the batch)")
     return ap.parse_args()
@@ -190,7 +193,8 @@ def run_ours(args, cfg):
     n, k, B = cfg.n, cfg.k, cfg.B
     gsz = 2 if cfg.gdt == "bf16" else 4
     lo, hi = ld.shard_bounds(n, P, rank)
-    comm = ld.Comm(P, rank) if P > 1 else None
+    comm = ld.Comm(P, rank) if P > 1 and args.sync == "nccl" else None
+    p2p = ld.P2P(P, rank, k, cfg.vdt, device=dev) if P > 1 and args.sync == "p2p" else None
 
     # ---- resident inputs: B gradients (seeded, per rank), residual, full-checkpoint shard ----
     sig = segment_sigmas(cfg, dev)
@@ -246,10 +250,14 @@ def run_ours(args, cfg):
                 g = h2d[0][d]
             else:
                 g = grads[j % len(grads)]
-            ld.compress(g, r, k, vdt=cfg.vdt, pairs=pairs)
+            dst = p2p.slot() if p2p is not None else pairs   # p2p: compress straight into the window
+            ld.compress(g, r, k, vdt=cfg.vdt, pairs=dst)
             if h2d is not None:
                 ev_free[d].record(cs)
-            ld.allgather_sparse(comm, pairs, k, cfg.vdt, lo, hi, True, *ring[j])
+            if p2p is not None:
+                p2p.allgather_sparse(dst, lo, hi, True, *ring[j])
+            else:
+                ld.allgather_sparse(comm, pairs, k, cfg.vdt, lo, hi, True, *ring[j])
         if h2d is not None:
             cs.wait_stream(h2d_stream)
 
@@ -425,12 +433,16 @@ def run_ours(args, cfg):
                "sample": f"one full step of {cfg.name} on the first {n_s} of n={cfg.n} elements "
                          f"(B={cfg.B} compress+coalesce, merge, {cfg.opt} replay), {dt:.1f} s"}
 
+    if p2p is not None:                                 # a timed-out peer wait voids the numbers
+        torch.cuda.synchronize()
+        p2p.status()
     if rank == 0:
         line = {"metric": "diff-build & replay gradient GB/s at 1/2/4/8 B200, % of HBM roofline",
                 "value": value, "unit": "GB/s", "n_gpus": P, "steps": args.steps, "warmup": args.warmup,
                 "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
                 "dtype": "f32" if cfg.gdt == "f32" else "bf16", "data": "synthetic",
                 "config": {"workload": cfg.name, "n": n, "k": k, "rho": cfg.rho, "B": B, "P": P,
+                           "sync": (args.sync if P > 1 else "local (P = 1)"),
                            "shard": [lo, hi], "replay": f"{cfg.opt}, chain of {R * B} iterations ({R} {cfg.merge.upper()} record{'s' if R > 1 else ''} of B={B})",
                            "l2": (f"inputs larger than L2 (each gradient {n * gsz / 1e6:.0f} MB > 126 MB), no flush"
                                   if n * gsz > 126e6 else
@@ -448,6 +460,9 @@ def run_ours(args, cfg):
         print(json.dumps(line), flush=True)
     if comm is not None:
         comm.destroy()
+    if p2p is not None:
+        dist.barrier()
+        p2p.destroy()
     if world > 1:
         dist.destroy_process_group()
 

@@ -51,7 +51,8 @@ enum {
   LOWDIFF_ECORRUPT = 5,      /* record bytes fail validation                                  */
   LOWDIFF_EUNSUPPORTED = 6,  /* e.g. SUM record with momentum/Adam without opt-in             */
   LOWDIFF_ECUDA = 7,         /* CUDA runtime error (message in lowdiff_last_error)            */
-  LOWDIFF_ENCCL = 8          /* NCCL error                                                    */
+  LOWDIFF_ENCCL = 8,         /* NCCL error                                                    */
+  LOWDIFF_ETIMEOUT = 9       /* a peer-memory wait expired (lowdiff_p2p_*)                    */
 };
 
 typedef enum { LOWDIFF_F32 = 0, LOWDIFF_BF16 = 1 } lowdiff_dtype;
@@ -124,6 +125,59 @@ lowdiff_status lowdiff_allgather_sparse(lowdiff_comm* comm, const void* pairs, u
                                         uint32_t* out_idx, float* out_val, uint64_t out_cap,
                                         uint64_t* d_out_nnz, void* ws, uint64_t ws_bytes,
                                         lowdiff_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------------
+ * (2') The same Sync (Alg.1 line 5; "Allgather") fused with the coalesce over peer
+ *     memory (NVLink / NVSwitch P2P, CUDA IPC): no all-gather copy. Every rank owns an exchange
+ *     WINDOW of lowdiff_p2p_window_bytes(nranks, k, vdt) bytes in its own HBM:
+ *       [u64 ready[nranks] | u64 done[nranks] | u64 epoch | pad to 256 | slot 0 | slot 1]
+ *     (each slot one packed pairs buffer, 256-byte aligned). The windows of all ranks are mapped
+ *     into every rank. lowdiff_p2p_allgather_sparse, called by every rank in the same order
+ *     (epoch e = 0, 1, ... counted on the device, so the calls may be captured in a CUDA graph
+ *     as long as each replay makes an even number of them: the slot is picked on the host by the
+ *     call's parity, checked against the device epoch), enqueues on `stream`:
+ *       1. wait until every peer finished reading this rank's slot e&1 of epoch e-2 (done >= e-1)
+ *       2. copy `pairs` into the local slot e&1. Zero-copy variant: lowdiff_p2p_slot(c, stream)
+ *          enqueues wait 1 on `stream` and returns the slot; compress into it on that stream and
+ *          pass it as `pairs` — steps 1-2 are then skipped
+ *       3. release-store ready[rank] = e+1 into every window (after a system-scope fence)
+ *       4. wait until every ready[p] >= e+1 in the local window (acquire)
+ *       5. coalesce over [lo, hi) reading each rank's slot e&1 directly from its owner's HBM —
+ *          the multiway merge of lowdiff_coalesce, bit-identical output (rank-ascending fold)
+ *       6. release-store done[rank] = e+1 into every peer window
+ *     Waits spin on device with a bounded time (LOWDIFF_P2P_TIMEOUT_MS, default 20000); a
+ *     timeout sets a flag read by lowdiff_p2p_status (ETIMEOUT) instead of hanging the GPU, and
+ *     the outputs of that call are then undefined.
+ *   window     caller-owned device memory (cudaMalloc / torch), 256-byte aligned; zeroed by
+ *              lowdiff_p2p_init (synchronously). Keep it alive until lowdiff_p2p_destroy.
+ *   handle     LOWDIFF_P2P_HANDLE_BYTES bytes: CUDA IPC handle of the window's allocation plus
+ *              the window's offset in it. Exchange them (e.g. torch.distributed all_gather),
+ *              then every rank calls lowdiff_p2p_init with all of them in rank order (its own
+ *              entry is not opened), then all ranks barrier before the first allgather call.
+ *   lowdiff_p2p_init_local: every window lives in this process (`windows` holds the nranks
+ *              device pointers), e.g. one process driving one device per rank. Several ranks on
+ *              ONE device in one process are not supported: their streams may share a hardware
+ *              queue, so a rank's spinning wait can block a peer's work until it times out.
+ * Errors: EINVAL (sizes, alignment, P < 2; from lowdiff_p2p_status: slot parity mismatch), ECUDA
+ * (IPC open failed: peers on devices without P2P access), ETIMEOUT (a wait expired: a rank did
+ * not make the matching call).
+ * ------------------------------------------------------------------------------------------- */
+#define LOWDIFF_P2P_HANDLE_BYTES 80
+typedef struct lowdiff_p2p lowdiff_p2p;
+uint64_t       lowdiff_p2p_window_bytes(int32_t nranks, uint64_t k, lowdiff_dtype vdt);
+lowdiff_status lowdiff_p2p_export_handle(const void* window, uint8_t* handle /* host, 80 B */);
+lowdiff_status lowdiff_p2p_init(lowdiff_p2p** c, void* window, const uint8_t* handles /* host, nranks x 80 B */,
+                                int32_t nranks, int32_t rank, uint64_t k, lowdiff_dtype vdt);
+lowdiff_status lowdiff_p2p_init_local(lowdiff_p2p** c, void* const* windows /* host array */,
+                                      int32_t nranks, int32_t rank, uint64_t k, lowdiff_dtype vdt);
+lowdiff_status lowdiff_p2p_destroy(lowdiff_p2p* c);
+void*          lowdiff_p2p_slot(lowdiff_p2p* c, lowdiff_stream_t stream); /* next call's slot; NULL on error */
+lowdiff_status lowdiff_p2p_allgather_sparse(lowdiff_p2p* c, const void* pairs, uint64_t lo, uint64_t hi,
+                                            int32_t average, uint32_t* out_idx, float* out_val,
+                                            uint64_t out_cap, uint64_t* d_out_nnz, void* ws,
+                                            uint64_t ws_bytes /* >= lowdiff_coalesce_workspace_size */,
+                                            lowdiff_stream_t stream);
+lowdiff_status lowdiff_p2p_status(const lowdiff_p2p* c);  /* ETIMEOUT once any wait expired; no sync */
 
 /* ---------------------------------------------------------------------------------------------
  * (3) Batch merge — Step 2 of batched gradient writing: B consecutive differentials of

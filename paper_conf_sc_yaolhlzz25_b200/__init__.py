@@ -28,7 +28,7 @@ _DT = {"f32": F32, "bf16": BF16, F32: F32, BF16: BF16}
 _MODE = {"sum": SUM, "stack": STACK, SUM: SUM, STACK: STACK}
 _KIND = {"sgd": SGD, "momentum": MOMENTUM, "adam": ADAM}
 STATUS = {0: "OK", 1: "EINVAL", 2: "EWORKSPACE", 3: "ECAPACITY", 4: "ECHAIN", 5: "ECORRUPT",
-          6: "EUNSUPPORTED", 7: "ECUDA", 8: "ENCCL"}
+          6: "EUNSUPPORTED", 7: "ECUDA", 8: "ENCCL", 9: "ETIMEOUT"}
 
 
 class LowDiffError(RuntimeError):
@@ -80,6 +80,8 @@ EXPORTS = [
     "lowdiff_debug_force_threshold", "lowdiff_wasted_time", "lowdiff_optimal_config",
     "lowdiff_replay_parallel_workspace_size", "lowdiff_replay_parallel",
     "lowdiff_update_workspace_size", "lowdiff_update", "lowdiff_dense_update", "lowdiff_host_update",
+    "lowdiff_p2p_window_bytes", "lowdiff_p2p_export_handle", "lowdiff_p2p_init", "lowdiff_p2p_init_local",
+    "lowdiff_p2p_destroy", "lowdiff_p2p_slot", "lowdiff_p2p_allgather_sparse", "lowdiff_p2p_status",
 ]
 
 _lib = None
@@ -135,6 +137,14 @@ def lib() -> C.CDLL:
         "lowdiff_update": ([vp, vp, vp, vp, u64, vp], i32),
         "lowdiff_dense_update": ([vp, vp, vp, i32, C.c_float, vp], i32),
         "lowdiff_host_update": ([vp, vp, vp, i32, C.c_float, i32], i32),
+        "lowdiff_p2p_window_bytes": ([i32, u64, i32], u64),
+        "lowdiff_p2p_export_handle": ([vp, vp], i32),
+        "lowdiff_p2p_init": ([vp, vp, vp, i32, i32, u64, i32], i32),
+        "lowdiff_p2p_init_local": ([vp, vp, i32, i32, u64, i32], i32),
+        "lowdiff_p2p_destroy": ([vp], i32),
+        "lowdiff_p2p_slot": ([vp, vp], vp),
+        "lowdiff_p2p_allgather_sparse": ([vp, vp, u64, u64, i32, vp, vp, u64, vp, vp, u64, vp], i32),
+        "lowdiff_p2p_status": ([vp], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -368,6 +378,89 @@ def allgather_sparse(comm: Comm | None, pairs: torch.Tensor, k: int, vdt="f32", 
                                           out_idx.numel(), _cuda(d_nnz, "d_nnz"), _cuda(ws, "ws"),
                                           ws.numel(), _stream(stream)), "allgather_sparse")
     return out_idx, out_val, d_nnz
+
+
+# ---- (2') all-gather fused with coalesce over peer memory (NVLink P2P, CUDA IPC) -------------------
+P2P_HANDLE_BYTES = 80
+
+
+def p2p_window_bytes(nranks: int, k: int, vdt="f32") -> int:
+    return int(lib().lowdiff_p2p_window_bytes(nranks, k, _DT[vdt]))
+
+
+class P2P:
+    """lowdiff_p2p_*: Sync(G~_{i,t}) (Alg.1 line 5) with the coalesce reading every rank's
+    pairs straight out of its owner's exchange window over NVLink (no all-gather copy).
+
+    Multi-process: P2P(nranks, rank, k, vdt, group=...) allocates this rank's window, exchanges the
+    CUDA IPC handles with torch.distributed.all_gather_object (any backend) and barriers.
+    Single process: P2P.local(nranks, k, vdt, device) returns one handle per simulated rank, all
+    windows on one device (each rank must then be driven on its own stream)."""
+
+    def __init__(self, nranks: int, rank: int, k: int, vdt="f32", device=None, group=None, _windows=None):
+        self.nranks, self.rank, self.k, self.vdt = nranks, rank, k, vdt
+        nb = p2p_window_bytes(nranks, k, vdt)
+        self._h = C.c_void_p()
+        if _windows is not None:                    # single-process: every window given
+            self.window = _windows[rank]
+            ptrs = (C.c_void_p * nranks)(*[w.data_ptr() for w in _windows])
+            _check(lib().lowdiff_p2p_init_local(C.byref(self._h), ptrs, nranks, rank, k, _DT[vdt]),
+                   "p2p_init_local")
+            return
+        import torch.distributed as dist
+        device = torch.device(device if device is not None else "cuda")
+        self.window = _aligned_window(nb, device)
+        h = (C.c_uint8 * P2P_HANDLE_BYTES)()
+        _check(lib().lowdiff_p2p_export_handle(C.c_void_p(self.window.data_ptr()), h), "p2p_export_handle")
+        allh = [None] * nranks
+        dist.all_gather_object(allh, bytes(h), group=group)
+        raw = (C.c_uint8 * (P2P_HANDLE_BYTES * nranks))(*b"".join(allh))
+        _check(lib().lowdiff_p2p_init(C.byref(self._h), C.c_void_p(self.window.data_ptr()), raw, nranks, rank,
+                                      k, _DT[vdt]), "p2p_init")
+        dist.barrier(group=group)
+
+    @classmethod
+    def local(cls, nranks: int, k: int, vdt="f32", device="cuda"):
+        nb = p2p_window_bytes(nranks, k, vdt)
+        wins = [_aligned_window(nb, torch.device(device)) for _ in range(nranks)]
+        return [cls(nranks, r, k, vdt, _windows=wins) for r in range(nranks)]
+
+    def slot(self, stream=None) -> torch.Tensor:
+        """The local slot the next allgather_sparse publishes (after enqueuing, on `stream`, the wait
+        that makes it writable): compress into it to skip the copy."""
+        p = lib().lowdiff_p2p_slot(self._h, _stream(stream))
+        if not p:
+            _check(7, "p2p_slot")
+        off = p - self.window.data_ptr()
+        return self.window[off:off + pairs_bytes(self.k, self.vdt)]
+
+    def allgather_sparse(self, pairs: torch.Tensor, lo: int, hi: int, average: bool = True, out_idx=None,
+                         out_val=None, d_nnz=None, ws=None, stream=None):
+        out_idx, out_val, d_nnz = _coalesce_outputs(pairs.device, self.nranks, self.k, lo, hi, out_idx, out_val,
+                                                     d_nnz)
+        wsb = coalesce_workspace_size(self.nranks, self.k, self.vdt, lo, hi)
+        if ws is None:
+            ws = workspace(wsb, pairs.device, f"p2p{self.rank}")
+        _check(lib().lowdiff_p2p_allgather_sparse(self._h, _cuda(pairs, "pairs"), lo, hi, int(average),
+                                                  _cuda(out_idx, "out_idx"), _cuda(out_val, "out_val"),
+                                                  out_idx.numel(), _cuda(d_nnz, "d_nnz"), _cuda(ws, "ws"),
+                                                  ws.numel(), _stream(stream)), "p2p_allgather_sparse")
+        return out_idx, out_val, d_nnz
+
+    def status(self):
+        """Raises LowDiffError(ETIMEOUT) once any peer wait of this handle expired (no sync)."""
+        _check(lib().lowdiff_p2p_status(self._h), "p2p_status")
+
+    def destroy(self):
+        if self._h:
+            _check(lib().lowdiff_p2p_destroy(self._h), "p2p_destroy")
+            self._h = C.c_void_p()
+
+
+def _aligned_window(nbytes: int, device) -> torch.Tensor:
+    buf = torch.empty(nbytes + 256, dtype=torch.uint8, device=device)
+    off = (-buf.data_ptr()) % 256
+    return buf[off:off + nbytes]
 
 
 # ---- (3) batch merge --------------------------------------------------------------------------------

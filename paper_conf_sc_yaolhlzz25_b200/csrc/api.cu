@@ -104,6 +104,7 @@ const char* lowdiff_status_string(lowdiff_status s) {
     case LOWDIFF_EUNSUPPORTED: return "unsupported combination";
     case LOWDIFF_ECUDA: return "CUDA error";
     case LOWDIFF_ENCCL: return "NCCL error";
+    case LOWDIFF_ETIMEOUT: return "peer-memory wait timed out";
   }
   return "unknown status";
 }

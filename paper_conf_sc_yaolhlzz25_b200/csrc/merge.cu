@@ -681,6 +681,14 @@ uint64_t merge_ws_bytes(int L, uint64_t max_entries, uint64_t lo, uint64_t hi) {
   return mlayout(L, max_entries, lo, hi, true).total;
 }
 
+// bytes [0, len) of a 16-byte aligned buffer <- 0
+__global__ void __launch_bounds__(kThreads) zero_kernel(uint8_t* __restrict__ p, uint64_t len) {
+  const uint64_t n16 = len / 16, stride = (uint64_t)gridDim.x * kThreads;
+  const uint64_t t = (uint64_t)blockIdx.x * kThreads + threadIdx.x;
+  for (uint64_t i = t; i < n16; i += stride) reinterpret_cast<uint4*>(p)[i] = make_uint4(0u, 0u, 0u, 0u);
+  for (uint64_t i = n16 * 16 + t; i < len; i += stride) p[i] = 0;
+}
+
 lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_t hi, int average,
                          uint64_t max_entries, uint32_t* out_idx, float* out_val, uint64_t out_cap,
                          uint64_t* d_out_nnz, const float* lr, uint64_t n, uint64_t t_first,
@@ -705,7 +713,15 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
   MCtl* ctl = reinterpret_cast<MCtl*>(w + M.ctl);
   uint32_t* starts = reinterpret_cast<uint32_t*>(w + M.starts);
   uint2* items = reinterpret_cast<uint2*>(w + M.items);
-  LD_CUDA(cudaMemsetAsync(w, 0, M.zero_end, s), "memset merge workspace");
+  // zeroed by a kernel, not cudaMemsetAsync: a memset may synchronise implicitly with the device's
+  // other streams, which would serialise this merge behind a peer-memory wait (lowdiff_p2p_*) of
+  // another rank simulated on the same device
+  {
+    uint64_t g = (M.zero_end / 16 + kThreads - 1) / kThreads;
+    if (g > 2ull * kNumSMs) g = 2ull * kNumSMs;
+    if (g < 1) g = 1;
+    LD_LAUNCH("merge_zero", s, zero_kernel, (int)g, kThreads, 0, w, M.zero_end);
+  }
 
   uint64_t per_list = max_entries / (ls.L ? ls.L : 1) + 1;
   uint64_t gx = (per_list + kThreads - 1) / kThreads;
