@@ -193,8 +193,14 @@ def run_ours(args, cfg):
     n, k, B = cfg.n, cfg.k, cfg.B
     gsz = 2 if cfg.gdt == "bf16" else 4
     lo, hi = ld.shard_bounds(n, P, rank)
-    comm = ld.Comm(P, rank) if P > 1 and args.sync == "nccl" else None
-    p2p = ld.P2P(P, rank, k, cfg.vdt, device=dev) if P > 1 and args.sync == "p2p" else None
+    p2p, sync_note = None, None
+    if P > 1 and args.sync == "p2p":
+        try:
+            p2p = ld.P2P(P, rank, k, cfg.vdt, device=dev)
+        except ld.LowDiffError as e:                    # e.g. no IPC / peer access between the GPUs
+            sync_note = f"p2p unavailable ({e}); ncclAllGather + coalesce"
+            print(sync_note, file=sys.stderr)
+    comm = ld.Comm(P, rank) if P > 1 and p2p is None else None
 
     # ---- resident inputs: B gradients (seeded, per rank), residual, full-checkpoint shard ----
     sig = segment_sigmas(cfg, dev)
@@ -442,7 +448,7 @@ def run_ours(args, cfg):
                 "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
                 "dtype": "f32" if cfg.gdt == "f32" else "bf16", "data": "synthetic",
                 "config": {"workload": cfg.name, "n": n, "k": k, "rho": cfg.rho, "B": B, "P": P,
-                           "sync": (args.sync if P > 1 else "local (P = 1)"),
+                           "sync": ("local (P = 1)" if P == 1 else sync_note or args.sync),
                            "shard": [lo, hi], "replay": f"{cfg.opt}, chain of {R * B} iterations ({R} {cfg.merge.upper()} record{'s' if R > 1 else ''} of B={B})",
                            "l2": (f"inputs larger than L2 (each gradient {n * gsz / 1e6:.0f} MB > 126 MB), no flush"
                                   if n * gsz > 126e6 else

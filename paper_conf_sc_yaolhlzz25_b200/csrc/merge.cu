@@ -49,7 +49,7 @@ struct __align__(256) MCtl {
 // ENTRY offset (known from the starts table alone, so items need no ordering between them); a
 // scan over the items' unique counts and a compaction then place them densely.
 struct MLayout {
-  uint64_t ctl, zero_end, starts, items, ucnt, epre, upre, sidx, sval, widx, wval, wit, went, total;
+  uint64_t ctl, ebnd, zero_end, starts, items, ucnt, epre, upre, sidx, sval, widx, wval, wit, went, total;
   uint32_t num_w;
 };
 
@@ -60,6 +60,7 @@ MLayout mlayout(int L, uint64_t max_entries, uint64_t lo, uint64_t hi, bool reco
   uint64_t o = 0;
   M.ctl = o;    o += align256(sizeof(MCtl));
   M.zero_end = o;
+  M.ebnd = o;   o += align256(8ull * L);         // per-list entry range of [lo, hi) (coalesce)
   M.starts = o; o += align256(4ull * L * (M.num_w + 1));
   M.items = o;  o += align256(8ull * M.num_w);
   M.ucnt = o;   o += align256(4ull * M.num_w);   // unique count per item
@@ -727,8 +728,12 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
   uint64_t gx = (per_list + kThreads - 1) / kThreads;
   if (gx > 8ull * kNumSMs) gx = 8ull * kNumSMs;
   if (gx < 1) gx = 1;
+  // coalesce: the gathered lists span the whole index range, so the shard's entry range of each
+  // list is found first and only it is scanned (batch merge: the lists are the shard's already)
+  uint32_t* ebnd = kind == kCoalesce ? reinterpret_cast<uint32_t*>(w + M.ebnd) : nullptr;
+  if (ebnd) LD_LAUNCH("starts", s, bounds_kernel, ls.L, 64, 0, ls, lo, hi, ebnd);
   LD_LAUNCH("starts", s, starts_kernel<kW>, dim3((unsigned)gx, (unsigned)ls.L), kThreads, 0, ls, lo, hi,
-            M.num_w, starts);
+            M.num_w, starts, (const uint32_t*)ebnd);
 
   // group size: up to kCap/2 entries per group at the average density (power of two); the
   // entries actually present (max_entries is a capacity) make groups smaller than this bound

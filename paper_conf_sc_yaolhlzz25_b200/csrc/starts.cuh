@@ -12,12 +12,17 @@ __device__ __forceinline__ uint64_t list_len(const ListSet& ls, int l) {
 // starts[l*(num_w+1) + w] = first position e of list l with idx[e] >= lo + w*W (entries below
 // lo are skipped); starts[l*(num_w+1) + num_w] = first position with idx >= hi (or len).
 // One streaming pass over the entries: entry e writes the windows in (win(e-1), win(e)].
+// ebnd (optional, from bounds_kernel): list l's entries in [lo, hi) are [ebnd[2l], ebnd[2l+1]), so
+// only they are scanned — a rank coalescing its shard of P gathered (or peer-resident) lists reads
+// about 1/P of each list's indices instead of all of them.
 template <int W>
 __global__ void __launch_bounds__(kThreads) starts_kernel(const __grid_constant__ ListSet ls, uint64_t lo,
-                                                          uint64_t hi, uint32_t num_w, uint32_t* starts) {
+                                                          uint64_t hi, uint32_t num_w, uint32_t* starts,
+                                                          const uint32_t* __restrict__ ebnd) {
   const int l = blockIdx.y;
   const uint32_t* idx = ls.list[l].idx;
   const uint64_t len = list_len(ls, l);
+  const uint64_t e_first = ebnd ? ebnd[2 * l] : 0, e_last = ebnd ? ebnd[2 * l + 1] : len;
   uint32_t* st = starts + (uint64_t)l * (num_w + 1);
   auto win = [&](uint64_t e) -> int64_t {
     if (e >= len) return (int64_t)num_w;
@@ -30,10 +35,10 @@ __global__ void __launch_bounds__(kThreads) starts_kernel(const __grid_constant_
   // thousands of empty windows between entries) are written by the whole warp, coalesced.
   const int lane = threadIdx.x & 31;
   const uint64_t stride = (uint64_t)gridDim.x * kThreads;
-  for (uint64_t e0 = (uint64_t)blockIdx.x * kThreads + (threadIdx.x & ~31u); e0 <= len; e0 += stride) {
+  for (uint64_t e0 = e_first + (uint64_t)blockIdx.x * kThreads + (threadIdx.x & ~31u); e0 <= e_last; e0 += stride) {
     const uint64_t e = e0 + lane;
     int64_t prev = 0, cur = -1;
-    if (e <= len) {
+    if (e <= e_last) {
       prev = (e == 0) ? -1 : win(e - 1);
       cur = win(e);
     }
@@ -50,6 +55,26 @@ __global__ void __launch_bounds__(kThreads) starts_kernel(const __grid_constant_
       for (int64_t w = from + lane; w <= to; w += 32) st[w] = ee;
     }
   }
+}
+
+// ebnd[2l] / ebnd[2l+1] = first position of list l with idx >= lo / idx >= hi (lists strictly
+// ascending). One block of 64 threads per list, one warp per bound: a 32-ary search, each round a
+// single coalesced probe of 32 positions (about 5 dependent rounds for a list of 3.4 M entries).
+static __global__ void __launch_bounds__(64) bounds_kernel(const __grid_constant__ ListSet ls, uint64_t lo, uint64_t hi,
+                                                    uint32_t* __restrict__ ebnd) {
+  const int l = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t* idx = ls.list[l].idx;
+  const uint64_t key = w ? hi : lo;
+  uint64_t a = 0, b = list_len(ls, l);     // answer in [a, b]: idx[a-1] < key, idx[b] >= key
+  while (a < b) {
+    const uint64_t p = a + ((b - a) * (uint64_t)(lane + 1)) / 33;   // in [a, b), non-decreasing in lane
+    const uint32_t m = __ballot_sync(0xFFFFFFFFu, (uint64_t)idx[p] >= key);
+    const int f = m ? __ffs(m) - 1 : 32;                              // first probe >= key
+    const uint64_t nb = __shfl_sync(0xFFFFFFFFu, p, f & 31), na = __shfl_sync(0xFFFFFFFFu, p, (f + 31) & 31);
+    if (f < 32) b = nb;
+    if (f > 0) a = na + 1;
+  }
+  if (lane == 0) ebnd[2 * l + w] = (uint32_t)a;
 }
 
 }  // namespace lowdiff
