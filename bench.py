@@ -183,11 +183,15 @@ def run_ours(args, cfg):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if os.environ.get("LOWDIFF_BENCH_DEVICE") is not None:   # tests: several ranks on one GPU
+        local = int(os.environ["LOWDIFF_BENCH_DEVICE"])
     assert world == args.gpus or world == 1, "--gpus must match the torchrun world size"
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        # host plumbing only (barriers, the max-over-ranks time, the p2p handle exchange, the NCCL id
+        # broadcast): gloo; the data path never goes through torch.distributed
+        dist.init_process_group("gloo")
     build.build()
     P = world
     n, k, B = cfg.n, cfg.k, cfg.B
@@ -312,7 +316,7 @@ def run_ours(args, cfg):
         torch.cuda.synchronize()
         ms = e0.elapsed_time(e1)
         if world > 1:
-            t = torch.tensor([ms], device=dev)
+            t = torch.tensor([ms], dtype=torch.float64)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ms = float(t.item())
             dist.barrier()
