@@ -50,6 +50,9 @@ def parse_args():
     ap.add_argument("--sync", default="p2p", choices=["p2p", "nccl"],
                     help="N > 1: all-gather fused with the coalesce over peer memory (p2p, default) or "
                          "ncclAllGather + coalesce (nccl)")
+    ap.add_argument("--copy-sync", action="store_true",
+                    help="P = 1: run the (identity) coalesce into a separate ring slot instead of the "
+                         "zero-copy hand-off")
     ap.add_argument("--grad-pool", type=int, default=0,
                     help="distinct resident gradients cycled through (0 = one per iteration of the batch)")
     return ap.parse_args()
@@ -226,6 +229,14 @@ def run_ours(args, cfg):
     ring = [(torch.empty(cap, dtype=torch.int32, device=dev), torch.empty(cap, device=dev),
              torch.zeros(1, dtype=torch.int64, device=dev)) for _ in range(B)]
     pairs = torch.empty(ld.pairs_bytes(k, cfg.vdt), dtype=torch.uint8, device=dev)
+    # P = 1 with fp32 values: the Sync of one list is the identity (union of one list, fp32 / 1
+    # exact), so ring slot j IS iteration j's compressed pairs buffer — the Reusing Queue's
+    # zero-copy hand-off: compress writes into the slot, the merge reads it in place.
+    zero_copy = P == 1 and cfg.vdt == "f32" and not args.copy_sync
+    if zero_copy:
+        slots = [torch.empty(ld.pairs_bytes(k, cfg.vdt), dtype=torch.uint8, device=dev) for _ in range(B)]
+        d_k = torch.full((1,), k, dtype=torch.int64, device=dev)
+        ring = [ld.pairs_views(sl, k, cfg.vdt) + (d_k,) for sl in slots]
     rec_cap = ld.record_max_bytes(cfg.merge, B, B * cap)
     R = chain_records(cfg)                              # batch records per step (replay chain K = R*B)
     records = [torch.empty(rec_cap, dtype=torch.uint8, device=dev) for _ in range(R)]
@@ -261,10 +272,14 @@ def run_ours(args, cfg):
             else:
                 g = grads[j % len(grads)]
             dst = p2p.slot() if p2p is not None else pairs   # p2p: compress straight into the window
+            if zero_copy:
+                dst = slots[j]
             ld.compress(g, r, k, vdt=cfg.vdt, pairs=dst)
             if h2d is not None:
                 ev_free[d].record(cs)
-            if p2p is not None:
+            if zero_copy:
+                pass                                    # the slot already holds G~_t
+            elif p2p is not None:
                 p2p.allgather_sparse(dst, lo, hi, True, *ring[j])
             else:
                 ld.allgather_sparse(comm, pairs, k, cfg.vdt, lo, hi, True, *ring[j])
@@ -472,7 +487,8 @@ def run_ours(args, cfg):
                 "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
                 "dtype": "f32" if cfg.gdt == "f32" else "bf16", "data": "synthetic",
                 "config": {"workload": cfg.name, "n": n, "k": k, "rho": cfg.rho, "B": B, "P": P,
-                           "sync": ("local (P = 1)" if P == 1 else sync_note or args.sync),
+                           "sync": (("local (P = 1): zero-copy ring of compressed pairs" if zero_copy else
+                                     "local (P = 1): coalesce into the ring") if P == 1 else sync_note or args.sync),
                            "shard": [lo, hi], "replay": f"{cfg.opt}, chain of {R * B} iterations ({R} {cfg.merge.upper()} record{'s' if R > 1 else ''} of B={B})",
                            "l2": (f"inputs larger than L2 (each gradient {n * gsz / 1e6:.0f} MB > 126 MB), no flush"
                                   if n * gsz > 126e6 else
