@@ -30,7 +30,7 @@ from __future__ import annotations
 import numpy as np
 import torch
 
-from . import (LowDiffError, allgather_sparse, batch_merge, compress, k_for_density, pairs_bytes,
+from . import (LowDiffError, allgather_sparse, batch_merge, compress, k_for_density, pairs_bytes, pairs_views,
                record_max_bytes, replay, shard_bounds, stage_d2h, update)
 
 _STATE_KEYS = ("x", "m", "v")
@@ -65,9 +65,17 @@ class LowDiffLoop:
         # training stream right after the batch's last update, so stream order puts it before the
         # next batch's writes into the same slots.
         R = B if checkpoint else 1
-        self.slots = [(torch.empty(self.cap, dtype=torch.int32, device=dev),
-                       torch.empty(self.cap, dtype=torch.float32, device=dev),
-                       torch.zeros(1, dtype=torch.int64, device=dev)) for _ in range(R)]
+        # P = 1: the Sync of one list is the identity, so a slot IS the compressed pairs buffer
+        # (compress writes it; the update and the merge read it in place: views + a count of k)
+        self.zero_copy = world == 1
+        if self.zero_copy:
+            d_k = torch.full((1,), self.k, dtype=torch.int64, device=dev)
+            self.pair_slots = [torch.empty(pairs_bytes(self.k), dtype=torch.uint8, device=dev) for _ in range(R)]
+            self.slots = [pairs_views(p, self.k) + (d_k,) for p in self.pair_slots]
+        else:
+            self.slots = [(torch.empty(self.cap, dtype=torch.int32, device=dev),
+                           torch.empty(self.cap, dtype=torch.float32, device=dev),
+                           torch.zeros(1, dtype=torch.int64, device=dev)) for _ in range(R)]
         self.ring = []                                                  # G~ of the open batch
         self.pairs = torch.empty(pairs_bytes(self.k), dtype=torch.uint8, device=dev)
         if not checkpoint:
@@ -101,9 +109,12 @@ class LowDiffLoop:
             if self.t % self.full_every == 0:
                 self._full_checkpoint()
         idx, val, nnz = self.slots[self.t % len(self.slots)]
-        pairs = compress(grad, self.r, self.k, pairs=self.pairs)
-        allgather_sparse(self.comm, pairs, self.k, "f32", self.lo, self.hi, out_idx=idx, out_val=val,
-                         d_nnz=nnz)
+        if self.zero_copy:
+            compress(grad, self.r, self.k, pairs=self.pair_slots[self.t % len(self.slots)])
+        else:
+            pairs = compress(grad, self.r, self.k, pairs=self.pairs)
+            allgather_sparse(self.comm, pairs, self.k, "f32", self.lo, self.hi, out_idx=idx, out_val=val,
+                             d_nnz=nnz)
         g_t = (idx, val, nnz, self.cap, self.lr)
         update(self.state, self.opt, g_t)                               # live M_{t+1}
         self.t += 1
