@@ -55,6 +55,16 @@ def test_host_helpers_match_definitions():
             assert ld.record_size(mode, B, nnz, nent) == oracle.record_size(om, B, nnz, nent)
 
 
+def test_p2p_window_layout():
+    """Exchange window of the fused Sync (include/lowdiff.h (2')): u64 ready[P] | u64 done[P] |
+    u64 epoch, padded to 256 B, then two 256-B aligned slots of one packed pairs buffer each."""
+    a256 = lambda x: (x + 255) // 256 * 256
+    for P in (2, 3, 8, 64):
+        for k, vdt in ((1, "f32"), (2697, "f32"), (3_351_418, "bf16")):
+            assert ld.p2p_window_bytes(P, k, vdt) == a256(16 * P + 8) + 2 * a256(ld.pairs_bytes(k, vdt))
+    assert ld.p2p_window_bytes(65, 100) == 0 and ld.p2p_window_bytes(2, 0) == 0   # out of range
+
+
 def test_record_parse_reads_oracle_records():
     rng = np.random.default_rng(3)
     diffs = []
