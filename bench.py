@@ -229,10 +229,10 @@ def run_ours(args, cfg):
     ring = [(torch.empty(cap, dtype=torch.int32, device=dev), torch.empty(cap, device=dev),
              torch.zeros(1, dtype=torch.int64, device=dev)) for _ in range(B)]
     pairs = torch.empty(ld.pairs_bytes(k, cfg.vdt), dtype=torch.uint8, device=dev)
-    # P = 1 with fp32 values: the Sync of one list is the identity (union of one list, fp32 / 1
-    # exact), so ring slot j IS iteration j's compressed pairs buffer — the Reusing Queue's
+    # P = 1: the Sync of one list is the identity (union of one list, fp32(v) / 1 exact), so ring
+    # slot j IS iteration j's compressed pairs buffer — the Reusing Queue's
     # zero-copy hand-off: compress writes into the slot, the merge reads it in place.
-    zero_copy = P == 1 and cfg.vdt == "f32" and not args.copy_sync
+    zero_copy = P == 1 and not args.copy_sync        # (bf16 values: widened exactly by the merge)
     if zero_copy:
         slots = [torch.empty(ld.pairs_bytes(k, cfg.vdt), dtype=torch.uint8, device=dev) for _ in range(B)]
         d_k = torch.full((1,), k, dtype=torch.int64, device=dev)

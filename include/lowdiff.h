@@ -214,6 +214,14 @@ lowdiff_status lowdiff_batch_merge(const lowdiff_diff_view* diffs /* host [B] */
                                    uint64_t t_first, uint32_t nranks, void* d_record,
                                    uint64_t record_cap, uint64_t* d_record_bytes, void* ws,
                                    uint64_t ws_bytes, lowdiff_stream_t stream);
+/* Same, with the diffs' values in `vdt` (`val` then points to bf16 when vdt = BF16): each value is
+ * widened to fp32 exactly, so the record equals the one built from the coalesced fp32 lists. This
+ * lets a P = 1 ring slot be the compressed pairs buffer itself (zero-copy), bf16 too. */
+lowdiff_status lowdiff_batch_merge_ex(const lowdiff_diff_view* diffs, uint32_t B, lowdiff_merge_mode mode,
+                                      lowdiff_dtype vdt, uint64_t n, uint64_t lo, uint64_t hi, uint64_t t_first,
+                                      uint32_t nranks, void* d_record, uint64_t record_cap,
+                                      uint64_t* d_record_bytes, void* ws, uint64_t ws_bytes,
+                                      lowdiff_stream_t stream);
 
 /* ---------------------------------------------------------------------------------------------
  * (4) Stage — Step 1, `offload_to_cpu()` non-blocking.

@@ -82,6 +82,7 @@ EXPORTS = [
     "lowdiff_update_workspace_size", "lowdiff_update", "lowdiff_dense_update", "lowdiff_host_update",
     "lowdiff_p2p_window_bytes", "lowdiff_p2p_export_handle", "lowdiff_p2p_init", "lowdiff_p2p_init_local",
     "lowdiff_p2p_destroy", "lowdiff_p2p_slot", "lowdiff_p2p_allgather_sparse", "lowdiff_p2p_status",
+    "lowdiff_batch_merge_ex",
 ]
 
 _lib = None
@@ -117,6 +118,8 @@ def lib() -> C.CDLL:
         "lowdiff_record_size": ([i32, C.c_uint32, u64, u64], u64),
         "lowdiff_record_max_bytes": ([i32, C.c_uint32, u64], u64),
         "lowdiff_batch_merge_workspace_size": ([C.c_uint32, u64, u64, u64, vp], i32),
+        "lowdiff_batch_merge_ex": ([vp, C.c_uint32, i32, i32, u64, u64, u64, u64, C.c_uint32, vp, u64, vp, vp,
+                                    u64, vp], i32),
         "lowdiff_batch_merge": ([vp, C.c_uint32, i32, u64, u64, u64, u64, C.c_uint32, vp, u64, vp, vp,
                                  u64, vp], i32),
         "lowdiff_record_bytes": ([vp, u64, vp, vp], i32),
@@ -474,7 +477,8 @@ def batch_merge_workspace_size(B: int, max_entries: int, lo: int, hi: int) -> in
 def batch_merge(diffs, mode, n: int, lo: int, hi: int, t_first: int, nranks: int, record=None,
                 d_record_bytes=None, ws=None, stream=None):
     """Merge B differentials [(idx int32, val fp32, d_nnz int64[1], cap, lr), ...] (iteration order)
-    into one record (§4.2 Step 2). Returns (record uint8 tensor, d_record_bytes int64[1])."""
+    into one record (§4.2 Step 2). Returns (record uint8 tensor, d_record_bytes int64[1]).
+    bf16 `val` tensors (a P = 1 ring of compressed pairs buffers) go through lowdiff_batch_merge_ex."""
     B = len(diffs)
     views = (DiffView * B)()
     dev = diffs[0][0].device
@@ -491,10 +495,14 @@ def batch_merge(diffs, mode, n: int, lo: int, hi: int, t_first: int, nranks: int
     wsb = batch_merge_workspace_size(B, max_entries, lo, hi)
     if ws is None:
         ws = workspace(wsb, dev, "merge")
-    _check(lib().lowdiff_batch_merge(views, B, _MODE[mode], n, lo, hi, t_first, nranks,
-                                     _cuda(record, "record"), record.numel(),
-                                     _cuda(d_record_bytes, "d_record_bytes"), _cuda(ws, "ws"), ws.numel(),
-                                     _stream(stream)), "batch_merge")
+    vdts = {d[1].dtype for d in diffs}
+    if vdts not in ({torch.float32}, {torch.bfloat16}):
+        raise ValueError("diff values must all be float32 or all bfloat16")
+    vdt = BF16 if vdts == {torch.bfloat16} else F32
+    _check(lib().lowdiff_batch_merge_ex(views, B, _MODE[mode], vdt, n, lo, hi, t_first, nranks,
+                                        _cuda(record, "record"), record.numel(),
+                                        _cuda(d_record_bytes, "d_record_bytes"), _cuda(ws, "ws"), ws.numel(),
+                                        _stream(stream)), "batch_merge")
     return record, d_record_bytes
 
 

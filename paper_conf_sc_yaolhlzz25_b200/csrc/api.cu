@@ -294,6 +294,16 @@ lowdiff_status lowdiff_batch_merge(const lowdiff_diff_view* diffs, uint32_t B, l
                                    uint64_t n, uint64_t lo, uint64_t hi, uint64_t t_first, uint32_t nranks,
                                    void* d_record, uint64_t record_cap, uint64_t* d_record_bytes, void* ws,
                                    uint64_t ws_bytes, lowdiff_stream_t stream) {
+  return lowdiff_batch_merge_ex(diffs, B, mode, LOWDIFF_F32, n, lo, hi, t_first, nranks, d_record, record_cap,
+                                d_record_bytes, ws, ws_bytes, stream);
+}
+
+lowdiff_status lowdiff_batch_merge_ex(const lowdiff_diff_view* diffs, uint32_t B, lowdiff_merge_mode mode,
+                                      lowdiff_dtype vdt, uint64_t n, uint64_t lo, uint64_t hi, uint64_t t_first,
+                                      uint32_t nranks, void* d_record, uint64_t record_cap,
+                                      uint64_t* d_record_bytes, void* ws, uint64_t ws_bytes,
+                                      lowdiff_stream_t stream) {
+  if (vdt != LOWDIFF_F32 && vdt != LOWDIFF_BF16) return fail(LOWDIFF_EINVAL, "batch_merge: bad value dtype");
   if (!diffs || B == 0 || B > 255 || lo >= hi || hi > n || n >= (1ull << 31) ||
       (mode != LOWDIFF_MERGE_SUM && mode != LOWDIFF_MERGE_STACK))
     return fail(LOWDIFF_EINVAL, "batch_merge: bad B/mode/range");
@@ -310,7 +320,7 @@ lowdiff_status lowdiff_batch_merge(const lowdiff_diff_view* diffs, uint32_t B, l
   if (ws_bytes < wsz) return fail(LOWDIFF_EWORKSPACE, "batch_merge: workspace too small");
   ListSet* ls = new ListSet();
   ls->L = (int)B;
-  ls->bf16 = 0;
+  ls->bf16 = vdt == LOWDIFF_BF16;
   float lr[256];
   for (uint32_t j = 0; j < B; ++j) {
     ls->list[j].idx = diffs[j].idx;

@@ -775,8 +775,14 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
   else if (kind == kCoalesce)
     LD_LAUNCH(cls, s, (merge_kernel<kCoalesce, false>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
               ucnt, epre, sidx, sval, oit, oent, sparse_max, bitmap_min);
+  else if (kind == kMergeSum && ls.bf16)
+    LD_LAUNCH(cls, s, (merge_kernel<kMergeSum, true>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
+              ucnt, epre, sidx, sval, oit, oent, sparse_max, bitmap_min);
   else if (kind == kMergeSum)
     LD_LAUNCH(cls, s, (merge_kernel<kMergeSum, false>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
+              ucnt, epre, sidx, sval, oit, oent, sparse_max, bitmap_min);
+  else if (ls.bf16)
+    LD_LAUNCH(cls, s, (merge_kernel<kMergeStack, true>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
               ucnt, epre, sidx, sval, oit, oent, sparse_max, bitmap_min);
   else
     LD_LAUNCH(cls, s, (merge_kernel<kMergeStack, false>), grid, kThreads, 0, ls, lo, M.num_w, starts, items, ctl,
