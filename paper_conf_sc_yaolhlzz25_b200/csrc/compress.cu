@@ -26,6 +26,8 @@ namespace {
 
 constexpr int kTile = 4096;            // elements per streaming tile: 256 thr x 4 vectors x 4
 constexpr int kMaxSelectBlocks = 4 * 148;
+constexpr int kSmallThreads = 1024;             // small select: one CTA
+constexpr uint32_t kSmallMaxCand = 1u << 15;    // candidate counts it takes (above: the grid kernel)
 // digit p = (key >> shift(p)) & (bins(p) - 1): 12 + 10 + 9 bits of the 31-bit key
 __host__ __device__ constexpr int bins(int p) { return p == 0 ? 4096 : (p == 1 ? 1024 : 512); }
 __host__ __device__ constexpr int shift(int p) { return p == 0 ? 19 : (p == 1 ? 9 : 0); }
@@ -38,14 +40,14 @@ struct __align__(256) Ctl {
   uint32_t sel_ticket[3];
   uint32_t prefix;         // key bits above the current digit
   uint32_t kstar;          // the k-th largest key
-  uint32_t pad0;
+  uint32_t small_done;     // the one-CTA select did this call (the grid kernel then returns)
   uint64_t k_rem;          // rank still to find below the prefix
   uint64_t count_gt;       // elements with key above the prefix range
   uint64_t m;              // K*-ties to keep (lowest indices first)
 };
 
 struct Layout {
-  uint64_t ctl, hs, hc, h0, h1, h2, zero_end, tiles, cand_idx, cand_val, tloc, boff, total;
+  uint64_t ctl, hs, hc, h0, h1, h2, zero_end, tiles, cand_idx, cand_val, tloc, boff, seg, pj, total;
   uint32_t num_tiles, cap;
 };
 
@@ -67,6 +69,8 @@ Layout layout(uint64_t n, uint64_t k) {
   L.cand_val = o; o += align256(4ull * L.cap);
   L.tloc = o;     o += align256(8ull * L.num_tiles);   // per-tile (gt, eq) counts, then their scan
   L.boff = o;     o += align256(8ull * 3 * kMaxSelectBlocks);
+  L.seg = o;      o += align256(16ull * L.num_tiles);  // small select: P at each tile's segment ends
+  L.pj = o;       o += align256(8ull * (L.cap < kSmallMaxCand ? L.cap : kSmallMaxCand));   // P per position
   L.total = o;
   return L;
 }
@@ -572,6 +576,7 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
   cg::grid_group grid = cg::this_grid();
   __shared__ uint32_t sh[bins(0)];
   __shared__ uint64_t s_scan[kThreads / 32];
+  if (ctl->small_done) return;                     // the one-CTA select did this call (uniform)
   const uint32_t cc = ctl->cand_count;
   const uint32_t mode = (cc >= k && cc <= cap) ? 0u : 1u;
   const float* src = mode ? r : cand_val;
@@ -725,6 +730,207 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
   }
 }
 
+
+// ---- K1c': small problems (<= 2^15 candidates): the same select + ordered emission in ONE CTA ----
+// The grid kernel's ~10 dependent phases each pay a grid barrier; for a few thousand candidates
+// (C1) one CTA does every phase behind __syncthreads. Work is split by candidate-buffer position:
+//   digits : shared-memory histograms of the candidates (12 bits from the stream pass, 10, 9)
+//   S      : exclusive prefix P(j) over buffer positions of packed (key > K*, key == K*); a tile's
+//            candidates are one contiguous segment, so P at its first and one-past-last position
+//            bound its counts
+//   B      : exclusive scan of the per-tile counts in index order
+//   C      : candidate j of tile t: (# > K* before it) = tile offset + P_gt(j) - P_gt(seg start),
+//            likewise for ties; kept iff key > K* or a tie among the first m -> slot; rejected
+//            candidates get r = a back (the stream pass stored them as selected).
+__device__ __forceinline__ uint64_t small_block_scan(uint64_t x, uint64_t* smem, uint64_t* total) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint64_t incl = x;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint64_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+    if (lane >= o) incl += y;
+  }
+  if (lane == 31) smem[warp] = incl;
+  __syncthreads();
+  if (warp == 0) {
+    const uint64_t v = smem[lane];
+    uint64_t w = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint64_t y = __shfl_up_sync(0xFFFFFFFFu, w, o);
+      if (lane >= o) w += y;
+    }
+    smem[lane] = w - v;                            // exclusive warp offsets
+    if (lane == 31) smem[32] = w;
+  }
+  __syncthreads();
+  const uint64_t r = smem[warp] + incl - x;
+  *total = smem[32];
+  __syncthreads();
+  return r;
+}
+
+// the bin of the need-th largest key (1-based) of a shared-memory histogram
+template <int NB>
+__device__ __forceinline__ int small_find(const uint32_t* h, uint64_t need, uint64_t* above_out, uint64_t* smem) {
+  __shared__ int s_bin;
+  __shared__ uint64_t s_above;
+  constexpr int PER = NB >= kSmallThreads ? NB / kSmallThreads : 1;
+  const bool act = (int)threadIdx.x * PER < NB;
+  const int lo = NB - ((int)threadIdx.x + 1) * PER;
+  uint32_t c[PER];
+  uint64_t sum = 0;
+#pragma unroll
+  for (int q = 0; q < PER; ++q) {
+    c[q] = act ? h[lo + q] : 0u;
+    sum += c[q];
+  }
+  if (threadIdx.x == 0) { s_bin = -1; s_above = 0; }
+  uint64_t total;
+  uint64_t above = small_block_scan(sum, smem, &total);
+  if (act && above < need && above + sum >= need) {
+#pragma unroll
+    for (int q = PER - 1; q >= 0; --q) {
+      if (above + c[q] >= need) { s_bin = lo + q; s_above = above; break; }
+      above += c[q];
+    }
+  }
+  __syncthreads();
+  *above_out = s_bin < 0 ? total : s_above;
+  return s_bin;
+}
+
+template <bool VBF16>
+__global__ void __launch_bounds__(kSmallThreads, 1)
+select_small_kernel(float* __restrict__ r, uint64_t k, Ctl* ctl, const float* __restrict__ cand_val,
+                    const uint32_t* __restrict__ cand_idx, const uint2* __restrict__ tile_info,
+                    uint32_t num_tiles, uint32_t cap, const uint32_t* __restrict__ hc,
+                    uint64_t* __restrict__ toff, ulonglong2* __restrict__ seg, uint64_t* __restrict__ pj,
+                    uint8_t* __restrict__ pairs) {
+  const uint32_t cc = ctl->cand_count;
+  if (!(cc >= k && cc <= cap && cc <= kSmallMaxCand)) return;   // the grid kernel does this call
+  __shared__ uint32_t s_h0[bins(0)], s_h1[bins(1)], s_h2[bins(2)];
+  __shared__ uint64_t s_scan[33];
+  const uint32_t tid = threadIdx.x, lane = tid & 31;
+  for (int b = tid; b < bins(0); b += kSmallThreads) s_h0[b] = __ldcg(hc + b);
+  for (int b = tid; b < bins(1); b += kSmallThreads) s_h1[b] = 0;
+  for (int b = tid; b < bins(2); b += kSmallThreads) s_h2[b] = 0;
+  __syncthreads();
+  uint64_t need = k, above;
+  const uint32_t d0 = (uint32_t)small_find<bins(0)>(s_h0, need, &above, s_scan);
+  need -= above;
+  auto digit = [&](uint32_t* sh, int NBITS, uint32_t pfx, int pshift, int dshift) {
+    for (uint32_t jw = tid & ~31u; jw < cc; jw += kSmallThreads) {   // warp-uniform trip count
+      const uint32_t j = jw + lane;
+      const uint32_t key = j < cc ? mag_key(cand_val[j]) : 0xFFFFFFFFu;
+      const bool take = key != 0xFFFFFFFFu && (key >> pshift) == pfx;
+      const uint32_t act = __ballot_sync(0xFFFFFFFFu, take);
+      if (take) {                                  // lanes with the same bin: one shared atomic
+        const uint32_t bin = (key >> dshift) & ((1u << NBITS) - 1);
+        const uint32_t peers = __match_any_sync(act, bin);
+        if (lane == __ffs(peers) - 1) atomicAdd(&sh[bin], (uint32_t)__popc(peers));
+      }
+    }
+    __syncthreads();
+  };
+  digit(s_h1, 10, d0, shift(0), shift(1));
+  const uint32_t d1 = (uint32_t)small_find<bins(1)>(s_h1, need, &above, s_scan);
+  need -= above;
+  const uint32_t p1 = (d0 << 10) | d1;
+  digit(s_h2, 9, p1, shift(1), shift(2));
+  const uint32_t d2 = (uint32_t)small_find<bins(2)>(s_h2, need, &above, s_scan);
+  need -= above;
+  const uint32_t K = (p1 << 9) | d2;
+  const uint64_t m = need;                         // K*-ties to keep (lowest indices first)
+  if (tid == 0) { ctl->mode = 0; ctl->kstar = K; ctl->m = m; ctl->small_done = 1; }
+  auto flag = [&](uint32_t j) -> uint64_t {        // packed (key > K*, key == K*) of position j
+    const uint32_t key = mag_key(cand_val[j]);
+    return ((uint64_t)(key > K) << 32) | (uint64_t)(key == K);
+  };
+  // S: P(j) over buffer positions, chunks of kSmallThreads x 4; segment boundaries record P
+  constexpr int kU = 4;
+  uint64_t base = 0;
+  for (uint32_t c0 = 0; c0 < cc; c0 += kSmallThreads * kU) {
+    uint64_t f[kU], sum = 0;
+    uint32_t ti[kU];
+    const uint32_t jf = c0 + tid * kU;
+    const uint32_t tbefore = (jf == 0 || jf > cc) ? 0xFFFFFFFFu : cand_idx[jf - 1] / kTile;
+    const uint32_t tafter = jf + kU >= cc ? 0xFFFFFFFFu : cand_idx[jf + kU] / kTile;
+#pragma unroll
+    for (int u = 0; u < kU; ++u) {
+      const uint32_t j = jf + u;
+      f[u] = j < cc ? flag(j) : 0;
+      ti[u] = j < cc ? cand_idx[j] / kTile : 0xFFFFFFFFu;
+      sum += f[u];
+    }
+    uint64_t ctot;
+    uint64_t run = base + small_block_scan(sum, s_scan, &ctot);
+#pragma unroll
+    for (int u = 0; u < kU; ++u) {
+      const uint32_t j = jf + u;
+      if (j < cc) {
+        pj[j] = run;
+        const uint32_t tprev = u ? ti[u - 1] : tbefore;
+        const uint32_t tnext = u < kU - 1 ? ti[u + 1] : tafter;
+        if (tprev != ti[u]) seg[ti[u]].x = run;                     // P at the segment's start
+        if (tnext != ti[u]) seg[ti[u]].y = run + f[u];              // P one past its end
+      }
+      run += f[u];
+    }
+    base += ctot;
+  }
+  __syncthreads();
+  // B: exclusive scan of the per-tile (gt, eq) counts in tile order
+  auto tcount = [&](uint32_t t) -> uint64_t {
+    if (tile_info[t].y == 0) return 0;
+    const ulonglong2 sg = seg[t];
+    return sg.y - sg.x;
+  };
+  base = 0;
+  for (uint32_t c0 = 0; c0 < num_tiles; c0 += kSmallThreads * kU) {
+    uint64_t v[kU], sum = 0;
+#pragma unroll
+    for (int u = 0; u < kU; ++u) {
+      const uint32_t t = c0 + tid * kU + u;
+      v[u] = t < num_tiles ? tcount(t) : 0;
+      sum += v[u];
+    }
+    uint64_t ctot;
+    uint64_t run = base + small_block_scan(sum, s_scan, &ctot);
+#pragma unroll
+    for (int u = 0; u < kU; ++u) {
+      const uint32_t t = c0 + tid * kU + u;
+      if (t < num_tiles) toff[t] = run;
+      run += v[u];
+    }
+    base += ctot;
+  }
+  __syncthreads();
+  // C: emission
+  uint32_t* out_idx = reinterpret_cast<uint32_t*>(pairs);
+  uint8_t* out_val = pairs + pad16(4 * k);
+  if (tid < 16) {                                  // zero the 16-byte padding of both sections
+    const uint64_t ip = 4 * k, ie = pad16(4 * k);
+    if (ip + tid < ie) pairs[ip + tid] = 0;
+    const uint64_t vp = pad16(4 * k) + (VBF16 ? 2 : 4) * k, ve = pad16(4 * k) + pad16((VBF16 ? 2 : 4) * k);
+    if (vp + tid < ve) pairs[vp + tid] = 0;
+  }
+  for (uint32_t j = tid; j < cc; j += kSmallThreads) {
+    const float a = cand_val[j];
+    const uint32_t idx = cand_idx[j], t = idx / kTile, key = mag_key(a);
+    const uint64_t before = toff[t] + (pj[j] - seg[t].x);        // packed (# > K*, # == K*) before j
+    const uint64_t gtb = before >> 32, eqb = before & 0xFFFFFFFFull;
+    if (key > K || (key == K && eqb < m)) {
+      const uint64_t pos = gtb + (eqb < m ? eqb : m);
+      out_idx[pos] = idx;
+      if constexpr (VBF16) reinterpret_cast<__nv_bfloat16*>(out_val)[pos] = __float2bfloat16_rn(a);
+      else reinterpret_cast<float*>(out_val)[pos] = a;
+    } else {
+      r[idx] = a;                                  // a rejected candidate keeps all of a
+    }
+  }
+}
+
 int g_stream_blocks_f32 = 0, g_stream_blocks_bf16 = 0;
 uint32_t g_force_t = 0xFFFFFFFFu;       // test hook: override the sampled threshold
 
@@ -870,6 +1076,22 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
                     (void*)&tiles_c, (void*)&nt, (void*)&cap, (void*)&h0, (void*)&h1, (void*)&h2,
                     (void*)&hcand, (void*)&tloc, (void*)&boff, (void*)&pp};
     ProfScope prof("compress_select", s);
+    static int use_small = -1;
+    if (use_small < 0) {
+      const char* e = getenv("LOWDIFF_SELECT_SMALL");
+      use_small = e ? atoi(e) : 1;
+    }
+    if (use_small && 4 * k <= kSmallMaxCand) {   // a few thousand candidates: one CTA does it all
+      ulonglong2* seg = reinterpret_cast<ulonglong2*>(w + L.seg);
+      uint64_t* pj = reinterpret_cast<uint64_t*>(w + L.pj);
+      if (vdt == LOWDIFF_BF16)
+        select_small_kernel<true><<<1, kSmallThreads, 0, s>>>(rr, k, ctl, cval, cidx, tiles, nt, cap, hcand, tloc,
+                                                               seg, pj, pp);
+      else
+        select_small_kernel<false><<<1, kSmallThreads, 0, s>>>(rr, k, ctl, cval, cidx, tiles, nt, cap, hcand, tloc,
+                                                                seg, pj, pp);
+      note_launch();
+    }
     const void* fn = vdt == LOWDIFF_BF16 ? (const void*)select_kernel<true> : (const void*)select_kernel<false>;
     LD_CUDA(cudaLaunchCooperativeKernel(fn, sel_grid, kThreads, args, 0, s), "select launch");
     note_launch();
