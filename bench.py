@@ -446,8 +446,36 @@ def run_ours(args, cfg):
         torch.cuda.synchronize()
         return e0.elapsed_time(e1) / reps
     replay_h2d_ms = replay_from_host()
+
+    # ---- stage (a5): the D2H copies of the step's records on the copy engine, and the pinned peak ----
+    def stage_timing():
+        torch.cuda.synchronize()
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(R)]
+        for b in range(R):
+            ev[b][0].record(copy_stream)
+            ld.stage_d2h(records[b], rec_nb[b], staged[b], copy_stream)
+            ev[b][1].record(copy_stream)
+        copy_stream.synchronize()
+        st_ms = sum(a.elapsed_time(z) for a, z in ev)
+        probe = torch.empty(1 << 28, dtype=torch.uint8, device=dev)
+        host = torch.empty(1 << 28, dtype=torch.uint8, pin_memory=True)
+        a, z = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        host.copy_(probe, non_blocking=True)
+        a.record()
+        for _ in range(3):
+            host.copy_(probe, non_blocking=True)
+        z.record()
+        torch.cuda.synchronize()
+        peak = 3 * (1 << 28) / (a.elapsed_time(z) * 1e-3) / 1e9
+        del probe, host
+        nbs = sum(rec_nb)
+        return {"bytes_per_step": int(nbs), "ms_per_step": st_ms, "gbs": nbs / (st_ms * 1e-3) / 1e9 if st_ms else None,
+                "pcie_d2h_peak_gbs": peak, "engine": "copy stream (cudaMemcpyAsync D2H into pinned memory)",
+                "hidden": bool(st_ms < replay_prof_ms),
+                "hidden_basis": "the last record's copy overlaps the recovery replay that follows it in the step"}
     build_prof_ms = sum(v[0] for c, v in prof.items() if not c.startswith("replay")) / args.steps
     replay_prof_ms = sum(v[0] for c, v in prof.items() if c.startswith("replay")) / args.steps
+    stage = stage_timing()
 
     # ---- e2e: same metric through the public API with host buffers (pinned H2D of every gradient) ----
     e2e = None
@@ -506,7 +534,7 @@ def run_ours(args, cfg):
                 "timing": {"build_phase": "one CUDA graph per step" if graph is not None else "eager launches",
                            "profiled_ms_per_step": pms / args.steps,
                            "profiled": "separate pass, eager launches, CUDA events around every kernel"},
-                "roofline": roofline, "replay_roofline": replay_roof, "kernels": kernels, "cpu_baseline": cpu, "e2e": e2e,
+                "roofline": roofline, "replay_roofline": replay_roof, "stage": stage, "kernels": kernels, "cpu_baseline": cpu, "e2e": e2e,
                 "gpu_launches": int(launches), "clocks": clk}
         print(json.dumps(line), flush=True)
     if comm is not None:
