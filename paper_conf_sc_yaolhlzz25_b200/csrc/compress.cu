@@ -131,18 +131,13 @@ __device__ int find_bin_desc(const uint32_t* h, uint64_t need, uint64_t* above_o
 // per-call phase, so small parameter segments are represented in proportion (coarse contiguous
 // chunks over-/under-represent segments smaller than their spacing, which biased the tail).
 // Exhaustive mode (small n) visits every micro-chunk.
+// This thread's share of the sample: micro-chunks m = first, first + step, ... -> histogram sh.
 template <bool BF16>
-__global__ void __launch_bounds__(kThreads) sample_kernel(const void* g, const float* r, uint64_t n,
-                                                          uint64_t k, uint32_t num_micro, double stride,
-                                                          double phase, int exhaustive, Ctl* ctl,
-                                                          uint32_t* hs, uint32_t force_t) {
-  __shared__ uint32_t sh[bins(0)];
-  __shared__ uint64_t s_scan[kThreads / 32];
-  __shared__ bool s_last;
-  for (int b = threadIdx.x; b < bins(0); b += kThreads) sh[b] = 0;
-  __syncthreads();
+__device__ __forceinline__ void sample_accumulate(const void* g, const float* r, uint64_t n, uint32_t num_micro,
+                                                  double stride, double phase, int exhaustive, uint32_t* sh,
+                                                  uint32_t first, uint32_t step) {
   const uint64_t n8 = n / 8;
-  for (uint32_t m = blockIdx.x * kThreads + threadIdx.x; m < num_micro; m += gridDim.x * kThreads) {
+  for (uint32_t m = first; m < num_micro; m += step) {
     uint64_t c8 = exhaustive ? m : (uint64_t)(((double)m + phase) * stride);
     if (!exhaustive && c8 >= n8) c8 = n8 ? n8 - 1 : 0;
     const uint64_t i = c8 * 8;
@@ -160,21 +155,19 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(const void* g, const f
       for (uint64_t j = i; j < n; ++j) atomicAdd(&sh[mag_key(load_g1<BF16>(g, j) + r[j]) >> shift(0)], 1u);
     }
   }
-  __syncthreads();
-  for (int b = threadIdx.x; b < bins(0); b += kThreads)
-    if (sh[b]) atomicAdd(hs + b, sh[b]);
-  __threadfence();
-  __syncthreads();
-  if (threadIdx.x == 0) s_last = (atomicAdd(&ctl->sample_ticket, 1u) == gridDim.x - 1);
-  __syncthreads();
-  if (!s_last) return;
-  __threadfence();
-  // Need: exhaustive -> exactly k (threshold = the bin's lower edge: exact, >= k candidates);
-  // sampled -> 1.3 x the expected sample count above the k-th key (+8): the candidates land at
-  // ~1.3 k, >7 sigma above k for S >= 512 n / k. Within the 12.5 %-wide bin the threshold is
-  // placed by an exponential-density model fitted to this bin and the next one up (the tail
-  // density falls steeply, so a uniform model lands too high), then moved 10 % toward the lower
-  // edge as a safety margin.
+}
+
+// The threshold from the finished sample histogram hs (block-wide; every thread gets it).
+// Need: exhaustive -> exactly k (threshold = the bin's lower edge: exact, >= k candidates);
+// sampled -> 1.3 x the expected sample count above the k-th key (+8): the candidates land at
+// ~1.3 k, >7 sigma above k for S >= 512 n / k. Within the 12.5 %-wide bin the threshold is
+// placed by an exponential-density model fitted to this bin and the next one up (the tail
+// density falls steeply, so a uniform model lands too high), then moved 10 % toward the lower
+// edge as a safety margin.
+__device__ __forceinline__ uint32_t threshold_from_sample(const uint32_t* hs, uint64_t n, uint64_t k,
+                                                          uint32_t num_micro, int exhaustive, uint32_t force_t,
+                                                          uint64_t* s_scan) {
+  __shared__ uint32_t s_t;
   uint64_t S = exhaustive ? n : (uint64_t)num_micro * 8;
   uint64_t need = exhaustive ? k : (uint64_t)(1.3 * (double)k * (double)S / (double)n) + 8;
   uint64_t above;
@@ -198,10 +191,50 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(const void* g, const f
       if (off >= (1u << shift(0))) off = (1u << shift(0)) - 1;
       t += off;
     }
-    ctl->t_est = (force_t != 0xFFFFFFFFu) ? force_t : t;   // force_t: test hook
+    s_t = (force_t != 0xFFFFFFFFu) ? force_t : t;   // force_t: test hook
+  }
+  __syncthreads();
+  return s_t;
+}
+
+template <bool BF16>
+__global__ void __launch_bounds__(kThreads) sample_kernel(const void* g, const float* r, uint64_t n,
+                                                          uint64_t k, uint32_t num_micro, double stride,
+                                                          double phase, int exhaustive, Ctl* ctl,
+                                                          uint32_t* hs, uint32_t force_t) {
+  __shared__ uint32_t sh[bins(0)];
+  __shared__ uint64_t s_scan[kThreads / 32];
+  __shared__ bool s_last;
+  for (int b = threadIdx.x; b < bins(0); b += kThreads) sh[b] = 0;
+  __syncthreads();
+  sample_accumulate<BF16>(g, r, n, num_micro, stride, phase, exhaustive, sh, blockIdx.x * kThreads + threadIdx.x,
+                          gridDim.x * kThreads);
+  __syncthreads();
+  for (int b = threadIdx.x; b < bins(0); b += kThreads)
+    if (sh[b]) atomicAdd(hs + b, sh[b]);
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) s_last = (atomicAdd(&ctl->sample_ticket, 1u) == gridDim.x - 1);
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  const uint32_t t = threshold_from_sample(hs, n, k, num_micro, exhaustive, force_t, s_scan);
+  if (threadIdx.x == 0) {
+    ctl->t_est = t;
     ctl->k_rem = k;
   }
 }
+
+// Arguments of the sample when it runs inside the stream kernel (FUSED): one cooperative launch
+// samples, meets at a grid barrier, derives the threshold in every CTA and streams.
+struct SampleArgs {
+  uint64_t k;
+  uint32_t num_micro;
+  double stride, phase;
+  int exhaustive;
+  uint32_t* hs;
+  uint32_t force_t;
+};
 
 // End of a streaming tile (both stream kernels): the tile's candidates go to the buffer (if it has
 // room) and the residual is stored. A candidate that was recorded is stored as if it were selected
@@ -249,19 +282,37 @@ __device__ __forceinline__ void tile_tail(float (&a)[4][4], uint32_t flags, uint
 }
 
 // ---- K1b: the fused streaming pass ----------------------------------------------------------
-template <bool BF16>
+template <bool BF16, bool FUSED = false>
 __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict__ g,
                                                           float* __restrict__ r, uint64_t n,
                                                           uint32_t num_tiles, Ctl* ctl,
                                                           uint2* __restrict__ tile_info,
                                                           uint32_t* __restrict__ cand_idx,
                                                           float* __restrict__ cand_val, uint32_t cap,
-                                                          int vbf16, uint32_t* __restrict__ hc) {
+                                                          int vbf16, uint32_t* __restrict__ hc,
+                                                          SampleArgs sa) {
   __shared__ uint64_t s_scan[2][kThreads / 32];
   __shared__ uint32_t s_base[2];
   __shared__ uint32_t s_h[bins(0)];               // first-digit histogram of this CTA's candidates
   for (int j = threadIdx.x; j < bins(0); j += kThreads) s_h[j] = 0;
-  const uint32_t T = ctl->t_est;
+  uint32_t T;
+  if constexpr (FUSED) {                           // the sample, then a grid barrier, then T
+    __syncthreads();
+    sample_accumulate<BF16>(g, r, n, sa.num_micro, sa.stride, sa.phase, sa.exhaustive, s_h,
+                            blockIdx.x * kThreads + threadIdx.x, gridDim.x * kThreads);
+    __syncthreads();
+    for (int j = threadIdx.x; j < bins(0); j += kThreads)
+      if (s_h[j]) { atomicAdd(sa.hs + j, s_h[j]); s_h[j] = 0; }
+    cg::this_grid().sync();
+    T = threshold_from_sample(sa.hs, n, sa.k, sa.num_micro, sa.exhaustive, sa.force_t, s_scan[0]);
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      ctl->t_est = T;
+      ctl->k_rem = sa.k;
+    }
+    __syncthreads();
+  } else {
+    T = ctl->t_est;
+  }
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   int par = 0;
   for (uint32_t tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, par ^= 1) {
@@ -1003,12 +1054,29 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   if (sg > 2ull * kNumSMs) sg = 2ull * kNumSMs;
   const int sample_grid = (int)sg;
   uint32_t* hs = reinterpret_cast<uint32_t*>(w + L.hs);
-  if (gdt == LOWDIFF_BF16)
-    LD_LAUNCH("compress_sample", s, sample_kernel<true>, sample_grid, kThreads, 0, grad, residual, n,
-              k, micro, stride, phase, exhaustive, ctl, hs, g_force_t);
-  else
-    LD_LAUNCH("compress_sample", s, sample_kernel<false>, sample_grid, kThreads, 0, grad, residual,
-              n, k, micro, stride, phase, exhaustive, ctl, hs, g_force_t);
+  static int use_tma = -1, fuse_sample = -1;
+  if (use_tma < 0) {
+    const char* e = getenv("LOWDIFF_STREAM_TMA");
+    use_tma = e ? atoi(e) : 0;
+    e = getenv("LOWDIFF_FUSED_SAMPLE");           // 0 never, 1 always, 2 (default) small grids
+    fuse_sample = e ? atoi(e) : 2;
+  }
+  // fused: the sample runs at the start of the (then cooperative) stream kernel, behind one grid
+  // barrier, instead of as its own launch that ends in a one-CTA threshold step. Measured: it pays
+  // off when the stream grid is small (every tile in one wave: n <= resident CTAs x 4096, C1:
+  // compress 0.161 -> 0.130 ms per 8 calls); with the full 740-CTA grid (C2, C3) the barrier and
+  // the per-CTA threshold step cost as much as the separate launch.
+  const bool fused = !use_tma && (fuse_sample == 1 ||
+                                  (fuse_sample == 2 && L.num_tiles <= (uint32_t)stream_blocks(gdt == LOWDIFF_BF16)));
+  SampleArgs sa{k, micro, stride, phase, exhaustive, hs, g_force_t};
+  if (!fused) {
+    if (gdt == LOWDIFF_BF16)
+      LD_LAUNCH("compress_sample", s, sample_kernel<true>, sample_grid, kThreads, 0, grad, residual, n,
+                k, micro, stride, phase, exhaustive, ctl, hs, g_force_t);
+    else
+      LD_LAUNCH("compress_sample", s, sample_kernel<false>, sample_grid, kThreads, 0, grad, residual,
+                n, k, micro, stride, phase, exhaustive, ctl, hs, g_force_t);
+  }
 
   uint2* tiles = reinterpret_cast<uint2*>(w + L.tiles);
   uint32_t* cidx = reinterpret_cast<uint32_t*>(w + L.cand_idx);
@@ -1016,11 +1084,6 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   const bool bf = gdt == LOWDIFF_BF16;
   const int vbf = vdt == LOWDIFF_BF16 ? 1 : 0;
   uint32_t* hcand = reinterpret_cast<uint32_t*>(w + L.hc);
-  static int use_tma = -1;
-  if (use_tma < 0) {
-    const char* e = getenv("LOWDIFF_STREAM_TMA");
-    use_tma = e ? atoi(e) : 0;
-  }
   if (use_tma) {
     int grid = stream_tma_blocks(bf);
     if ((uint32_t)grid > L.num_tiles) grid = (int)L.num_tiles;
@@ -1034,12 +1097,21 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   } else {
     int grid = stream_blocks(bf);
     if ((uint32_t)grid > L.num_tiles) grid = (int)L.num_tiles;
-    if (bf)
+    if (fused) {                                   // co-resident by construction (occupancy grid)
+      uint32_t nt = L.num_tiles, cp = L.cap;
+      void* args[] = {(void*)&grad, (void*)&residual, (void*)&n, (void*)&nt, (void*)&ctl, (void*)&tiles,
+                      (void*)&cidx, (void*)&cval, (void*)&cp, (void*)&vbf, (void*)&hcand, (void*)&sa};
+      ProfScope prof("compress_stream", s);
+      const void* fn = bf ? (const void*)stream_kernel<true, true> : (const void*)stream_kernel<false, true>;
+      LD_CUDA(cudaLaunchCooperativeKernel(fn, grid, kThreads, args, 0, s), "stream launch");
+      note_launch();
+    } else if (bf) {
       LD_LAUNCH("compress_stream", s, stream_kernel<true>, grid, kThreads, 0, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand);
-    else
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, sa);
+    } else {
       LD_LAUNCH("compress_stream", s, stream_kernel<false>, grid, kThreads, 0, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, sa);
+    }
   }
 
   {
