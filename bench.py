@@ -229,6 +229,8 @@ def run_ours(args, cfg):
     ring = [(torch.empty(cap, dtype=torch.int32, device=dev), torch.empty(cap, device=dev),
              torch.zeros(1, dtype=torch.int64, device=dev)) for _ in range(B)]
     pairs = torch.empty(ld.pairs_bytes(k, cfg.vdt), dtype=torch.uint8, device=dev)
+    # the residual's own compress workspace: it carries the warm threshold state between calls
+    cws = torch.empty(ld.compress_workspace_size(n, k), dtype=torch.uint8, device=dev)
     # P = 1: the Sync of one list is the identity (union of one list, fp32(v) / 1 exact), so ring
     # slot j IS iteration j's compressed pairs buffer — the Reusing Queue's
     # zero-copy hand-off: compress writes into the slot, the merge reads it in place.
@@ -274,7 +276,7 @@ def run_ours(args, cfg):
             dst = p2p.slot() if p2p is not None else pairs   # p2p: compress straight into the window
             if zero_copy:
                 dst = slots[j]
-            ld.compress(g, r, k, vdt=cfg.vdt, pairs=dst)
+            ld.compress(g, r, k, vdt=cfg.vdt, pairs=dst, ws=cws)
             if h2d is not None:
                 ev_free[d].record(cs)
             if zero_copy:
@@ -368,14 +370,24 @@ def run_ours(args, cfg):
     clocks = ClockSampler(local)
     clocks.start()
     launches0 = ld.launch_count()
+    cc0 = ld.compress_counters(ws=cws)
     ms, rec_bytes = timed(args.steps, graph=graph)
+    cc1 = ld.compress_counters(ws=cws)
     launches = ld.launch_count() - launches0 + (graph_launches * args.steps if graph is not None else 0)
     clk = clocks.stop()
     # ---- profiled pass (same work, eager launches, CUDA events around every kernel) ----
     ld.profile_enable(True)
     pms, _ = timed(args.steps)
     ld.profile_enable(False)
-    prof = {c: ld.profile_query(c) for c in ("compress_stream", "compress_sample", "compress_select",
+    cc2 = ld.compress_counters(ws=cws)
+    # compress paths over both passes: 0 = warm first-pass candidates, 2 = rescan
+    # recovery inside the select, 1 = exact full-array select; counted on the device
+    paths = {"calls": cc2["calls"] - cc0["calls"], "rescans": cc2["rescans"] - cc0["rescans"],
+             "fallbacks": cc2["fallbacks"] - cc0["fallbacks"],
+             "timed": {q: cc1[q] - cc0[q] for q in ("calls", "rescans", "fallbacks")},
+             "since_start": {q: cc2[q] for q in ("calls", "rescans", "fallbacks", "nonfinite_calls")},
+             "last_candidates_per_k": cc2["last_candidates"] / k, "margin": cc2["delta"]}
+    prof = {c: ld.profile_query(c) for c in ("compress_stream", "compress_select",
                                              "coalesce", "starts", "merge", "merge_pack",
                                              "replay_dense", "replay_sparse")}
     ms_step = ms / args.steps
@@ -530,7 +542,8 @@ def run_ours(args, cfg):
                                                "step); replayed iterations/s = K / replay kernel time, and "
                                                "with the records copied H2D from pinned memory first "
                                                "(profiled pass, CUDA events)",
-                           "record_bytes": int(rec_bytes)},
+                           "record_bytes": int(rec_bytes),
+                           "compress_paths": paths},
                 "timing": {"build_phase": "one CUDA graph per step" if graph is not None else "eager launches",
                            "profiled_ms_per_step": pms / args.steps,
                            "profiled": "separate pass, eager launches, CUDA events around every kernel"},

@@ -84,10 +84,22 @@ lowdiff_status lowdiff_shard_bounds(uint64_t n, int32_t nranks, int32_t rank, ui
  *         vdt BF16: val = bf16_rne(a[S]);   residual <- a off S, a - fp32(val) on S (exact)
  *   grad      [n] gdt (F32 or BF16), read only.      residual [n] fp32, updated in place.
  *   pairs     lowdiff_pairs_bytes(k, vdt) bytes, written.   1 <= k <= n < 2^31.
- *   ws        lowdiff_compress_workspace_size(n, k) bytes; contents need not be preserved.
- * Errors: EINVAL (k, n, dtype, alignment), EWORKSPACE. The streaming pass is driven by a
- * sampled threshold; if it under- or over-shoots, an exact full-array path runs on device
- * (same result, more HBM traffic); nothing is reported to the host.
+ *   ws        lowdiff_compress_workspace_size(n, k) bytes, device, 16-byte aligned. Its first 256
+ *             bytes carry a per-residual threshold STATE between calls (the previous call's exact
+ *             k-th key, an adaptive margin, counters): pass the same ws for the same residual to
+ *             keep it warm. The state is a hint only — a fresh, foreign or garbage workspace reads as
+ *             "cold" (checked against n, k, the residual pointer and the dtypes) and the OUTPUT IS
+ *             IDENTICAL either way; the rest of ws is scratch.
+ * Execution: one streaming pass keeps every element whose key is >= T (T = the previous k-th key
+ *   lowered by the margin) as a candidate; one cooperative select finds the exact k-th key among
+ *   them and writes the pairs. If the candidates number < k (cold start, or the k-th key dropped
+ *   by more than the margin) or exceed the capacity (8k + 65536), the select recovers on device
+ *   with ONE rescan of the residual at a corrected threshold (from a stratified sample, resp. the
+ *   exact first-digit histogram of the candidates); only if that also misses does an exact
+ *   full-array select run. Paths and non-finite inputs are counted in the state:
+ *   lowdiff_compress_counters.
+ * Errors: EINVAL (k, n, dtype, alignment), EWORKSPACE. Non-finite a (Inf/NaN) are ordered by bit
+ *   pattern above every finite key (reading #4) and counted, not rejected.
  * ------------------------------------------------------------------------------------------- */
 lowdiff_status lowdiff_compress_workspace_size(uint64_t n, uint64_t k, uint64_t* bytes);
 lowdiff_status lowdiff_compress(const void* grad, lowdiff_dtype gdt, float* residual, uint64_t n,
@@ -384,14 +396,22 @@ lowdiff_status lowdiff_optimal_config(const lowdiff_config_model* m, double* f_s
  *     "merge_pack", "replay_dense", "replay_sparse", "starts".
  * ------------------------------------------------------------------------------------------- */
 uint64_t       lowdiff_launch_count(void);
-/* After a lowdiff_compress on `stream` with workspace `ws` (syncs the stream): out6 = {sampled
- * threshold key, candidates found, path (0 = candidate buffer, 1 = full-array fallback), k-th key,
- * ties kept, candidate capacity}. Diagnostics for tests and the bench. */
+/* After a lowdiff_compress on `stream` with workspace `ws` (syncs the stream): out6 = {first-pass
+ * threshold key, first-pass candidates found, path (0 = first-pass candidates, 2 = rescan
+ * candidates, 1 = full-array select), k-th key, ties kept, candidate capacity}. Diagnostics. */
 lowdiff_status lowdiff_compress_stats(const void* ws, uint64_t n, uint64_t k, lowdiff_stream_t stream,
                                       uint64_t* out6);
-/* Test hook: while enabled, every later lowdiff_compress uses `key` as its candidate threshold
- * instead of the sampled estimate (to force the exact full-array fallback in tests). */
+/* The threshold state of the residual `ws` was last used with (syncs `stream`): out8 =
+ * {calls, rescans (path 2), full-array fallbacks (path 1), calls that saw non-finite a, non-finite
+ * count of the last call, first-pass candidates of the last call, last k-th key, margin x 2^32}.
+ * All zero for a workspace never used by lowdiff_compress. Counters restart when the workspace
+ * moves to another residual / n / k. */
+lowdiff_status lowdiff_compress_counters(const void* ws, lowdiff_stream_t stream, uint64_t* out8);
+/* Test hooks: while enabled, every later lowdiff_compress uses `key` as its first-pass candidate
+ * threshold (lowdiff_debug_force_threshold: drives the rescan recovery) or as the rescan's
+ * threshold (lowdiff_debug_force_rescan_threshold: drives the exact full-array path). */
 lowdiff_status lowdiff_debug_force_threshold(int32_t enable, uint32_t key);
+lowdiff_status lowdiff_debug_force_rescan_threshold(int32_t enable, uint32_t key);
 lowdiff_status lowdiff_profile_enable(int32_t on);
 lowdiff_status lowdiff_profile_query(const char* name, double* total_ms, uint64_t* launches);
 

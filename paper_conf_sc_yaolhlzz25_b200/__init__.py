@@ -77,7 +77,8 @@ EXPORTS = [
     "lowdiff_batch_merge", "lowdiff_record_bytes", "lowdiff_stage_d2h", "lowdiff_record_parse",
     "lowdiff_replay_workspace_size", "lowdiff_replay", "lowdiff_launch_count",
     "lowdiff_profile_enable", "lowdiff_profile_query", "lowdiff_compress_stats",
-    "lowdiff_debug_force_threshold", "lowdiff_wasted_time", "lowdiff_optimal_config",
+    "lowdiff_debug_force_threshold", "lowdiff_debug_force_rescan_threshold", "lowdiff_compress_counters",
+    "lowdiff_wasted_time", "lowdiff_optimal_config",
     "lowdiff_replay_parallel_workspace_size", "lowdiff_replay_parallel",
     "lowdiff_update_workspace_size", "lowdiff_update", "lowdiff_dense_update", "lowdiff_host_update",
     "lowdiff_p2p_window_bytes", "lowdiff_p2p_export_handle", "lowdiff_p2p_init", "lowdiff_p2p_init_local",
@@ -132,6 +133,8 @@ def lib() -> C.CDLL:
         "lowdiff_profile_query": ([C.c_char_p, vp, vp], i32),
         "lowdiff_compress_stats": ([vp, u64, u64, vp, vp], i32),
         "lowdiff_debug_force_threshold": ([i32, C.c_uint32], i32),
+        "lowdiff_debug_force_rescan_threshold": ([i32, C.c_uint32], i32),
+        "lowdiff_compress_counters": ([vp, vp, vp], i32),
         "lowdiff_wasted_time": ([vp, f64, f64, vp], i32),
         "lowdiff_replay_parallel_workspace_size": ([vp, vp, C.c_uint32, vp], i32),
         "lowdiff_replay_parallel": ([vp, vp, vp, C.c_uint32, vp, u64, vp], i32),
@@ -656,18 +659,41 @@ def replay_parallel(state: dict, opt: dict, records, ws=None, stream=None) -> di
 
 
 # ---- instrumentation --------------------------------------------------------------------------------
-def compress_stats(n: int, k: int, device="cuda", stream=None) -> dict:
-    """Diagnostics of the last compress that used the cached workspace (syncs the stream)."""
-    ws = workspace(compress_workspace_size(n, k), device, "compress")
+def compress_stats(n: int, k: int, device="cuda", stream=None, ws=None) -> dict:
+    """Diagnostics of the last compress that used `ws` (default: the cached workspace; syncs).
+    path: 0 = first-pass candidates, 2 = rescan recovery, 1 = exact full-array select."""
+    if ws is None:
+        ws = workspace(compress_workspace_size(n, k), device, "compress")
     out = (C.c_uint64 * 6)()
     _check(lib().lowdiff_compress_stats(_cuda(ws, "ws"), n, k, _stream(stream), out), "compress_stats")
-    return dict(zip(("t_est", "candidates", "fallback", "kstar", "ties_kept", "capacity"), list(out)))
+    d = dict(zip(("t_est", "candidates", "path", "kstar", "ties_kept", "capacity"), list(out)))
+    d["fallback"] = int(d["path"] == 1)
+    d["rescan"] = int(d["path"] == 2)
+    return d
+
+
+def compress_counters(n: int = 0, k: int = 0, device="cuda", stream=None, ws=None) -> dict:
+    """The persistent threshold state of a compress workspace (syncs): calls, rescans, full-array
+    fallbacks, non-finite calls/count, last candidates, last k-th key, margin."""
+    if ws is None:
+        ws = workspace(compress_workspace_size(n, k), device, "compress")
+    out = (C.c_uint64 * 8)()
+    _check(lib().lowdiff_compress_counters(_cuda(ws, "ws"), _stream(stream), out), "compress_counters")
+    v = list(out)
+    return {"calls": v[0], "rescans": v[1], "fallbacks": v[2], "nonfinite_calls": v[3],
+            "last_nonfinite": v[4], "last_candidates": v[5], "kstar": v[6], "delta": v[7] / 2.0 ** 32}
 
 
 def debug_force_threshold(key: int | None):
-    """Test hook: force the compress candidate threshold (None restores the sampled estimate)."""
+    """Test hook: force the compress first-pass candidate threshold (None restores the default)."""
     _check(lib().lowdiff_debug_force_threshold(0 if key is None else 1, 0 if key is None else key),
            "debug_force_threshold")
+
+
+def debug_force_rescan_threshold(key: int | None):
+    """Test hook: force the threshold of the compress rescan recovery (None restores the default)."""
+    _check(lib().lowdiff_debug_force_rescan_threshold(0 if key is None else 1, 0 if key is None else key),
+           "debug_force_rescan_threshold")
 
 
 def launch_count() -> int:

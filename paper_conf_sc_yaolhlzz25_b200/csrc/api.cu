@@ -559,8 +559,18 @@ lowdiff_status lowdiff_replay_parallel(lowdiff_state* st, const lowdiff_opt* opt
 uint64_t lowdiff_launch_count(void) { return g_launches.load(); }
 
 lowdiff_status lowdiff_debug_force_threshold(int32_t enable, uint32_t key) {
-  compress_force_threshold(enable, key);
+  compress_force_threshold(0, enable, key);
   return LOWDIFF_OK;
+}
+
+lowdiff_status lowdiff_debug_force_rescan_threshold(int32_t enable, uint32_t key) {
+  compress_force_threshold(1, enable, key);
+  return LOWDIFF_OK;
+}
+
+lowdiff_status lowdiff_compress_counters(const void* ws, lowdiff_stream_t stream, uint64_t* out8) {
+  if (!ws || !out8) return fail(LOWDIFF_EINVAL, "compress_counters: null");
+  return compress_counters(ws, (cudaStream_t)stream, out8);
 }
 
 lowdiff_status lowdiff_compress_stats(const void* ws, uint64_t n, uint64_t k, lowdiff_stream_t stream,

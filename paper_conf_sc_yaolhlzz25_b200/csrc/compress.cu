@@ -2,15 +2,27 @@
 // error feedback, on sm_100a.
 //
 // Design: the only HBM-heavy step is one fused streaming pass
-//   a = g + r;  r <- a;  if |a| >= T_est: append (i, a) to a candidate buffer
-// which moves the algorithmic floor of 12n bytes (fp32 g) / 10n (bf16 g). T_est comes from a
-// small stratified sample of |g + r| (8-element micro-chunks, >= 512 n/k keys) so the
-// candidates number ~1.3-2 k. One cooperative kernel then does the rest: an exact 3-digit radix
-// select (12/10/9 bits of the 31-bit key) over the candidates finds the k-th key K* and the number
-// m of K*-ties to keep, and an ordered emission (per-tile counts, a scan over tiles, ballot
-// prefixes inside each tile) writes the k pairs in ascending index order and fixes r on S.
-// If the sample under- or over-shot (candidates < k or > capacity) the same kernel runs over the
-// full residual array instead (exact, ~+12n bytes; not observed on the synthetic workloads).
+//   a = g + r;  r <- a;  if |a| >= T: append (i, a) to a candidate buffer
+// which moves the algorithmic floor of 12n bytes (fp32 g) / 10n (bf16 g). The candidate threshold
+// T comes from the previous call's exact k-th key K*_prev, lowered by an adaptive margin delta
+// (persistent per-residual state kept in the workspace; a hint only — the result never depends on
+// it): in error-feedback steady state the k-th key moves by a fraction of a percent per iteration,
+// while the key density right below it piles up (every unselected element keeps accumulating
+// until it crosses the threshold), so a sampled estimate with a few percent of resolution is not
+// accurate enough there (305 of 1300 C3 calls fell back with the sample alone).
+// One cooperative kernel then does the rest: an exact 3-digit radix select (12/10/9 bits of the
+// 31-bit key) over the candidates finds K* and the number m of K*-ties to keep, and an ordered
+// emission (per-tile counts, a scan over tiles, ballot prefixes inside each tile) writes the k
+// pairs in ascending index order and fixes r on S.
+// Recovery, all inside the same select launch (no host round trip):
+//   * fewer than k candidates (the first call on a residual, or K* dropped by more than delta):
+//     a stratified sample of |g + r| gives a lower threshold T2;
+//   * more than the capacity: the stream pass's exact first-digit histogram of ALL candidates
+//     gives T2 = the lower edge of the k-th key's bin;
+//   then one rescan of the residual (4n bytes read; the first pass's recorded candidates are
+//   overlaid from the buffer) rebuilds the candidate set at T2. Only if that also misses does the
+//   exact full-array select run (~3 x 4n bytes). Every path gives the same bytes; the per-call path
+//   and counters are reported through lowdiff_compress_counters.
 // Nothing on this path is a dense contraction: no tensor cores.
 #include <stdio.h>
 
@@ -28,26 +40,43 @@ constexpr int kTile = 4096;            // elements per streaming tile: 256 thr x
 constexpr int kMaxSelectBlocks = 4 * 148;
 constexpr int kSmallThreads = 1024;             // small select: one CTA
 constexpr uint32_t kSmallMaxCand = 1u << 15;    // candidate counts it takes (above: the grid kernel)
+constexpr uint32_t kNoForce = 0xFFFFFFFFu;
 // digit p = (key >> shift(p)) & (bins(p) - 1): 12 + 10 + 9 bits of the 31-bit key
 __host__ __device__ constexpr int bins(int p) { return p == 0 ? 4096 : (p == 1 ? 1024 : 512); }
 __host__ __device__ constexpr int shift(int p) { return p == 0 ? 19 : (p == 1 ? 9 : 0); }
+constexpr uint32_t kNonFiniteBin = 0x7F800000u >> 19;   // first-digit bins >= this hold Inf/NaN keys
+
+// Persistent per-residual state (the first 256 bytes of the workspace; never cleared by a call).
+// It is valid only for the (n, k, residual, dtypes) it was written for; anything else (a fresh or
+// reused workspace) reads as "cold" and the call takes the recovery path once.
+constexpr uint64_t kStateMagic = 0x4C44435354415445ull;   // "LDCSTATE"
+struct __align__(256) State {
+  uint64_t magic, n, k, resid, tag;
+  uint32_t kstar;           // the previous call's exact k-th key
+  float delta;              // relative margin below it for the next threshold
+  uint64_t calls, rescans, fallbacks, nonfinite_calls, last_nonfinite;
+  uint32_t last_cand, last_path;
+};
+struct StateKey {
+  uint64_t n, k, resid, tag;
+};
+constexpr float kDeltaInit = 1.0f / 64, kDeltaMin = 1.0f / 8192, kDeltaMax = 0.5f;
 
 struct __align__(256) Ctl {
-  uint32_t t_est;          // candidates: key >= t_est
-  uint32_t mode;           // 0 = candidate buffer, 1 = full residual array
+  uint32_t t_est;          // the first pass's threshold: candidates have key >= t_est
+  uint32_t mode;           // path: 0 = first-pass candidates, 2 = rescan candidates, 1 = full array
   uint32_t cand_count;     // candidates found by the streaming pass (may exceed capacity)
-  uint32_t sample_ticket;
-  uint32_t sel_ticket[3];
-  uint32_t prefix;         // key bits above the current digit
+  uint32_t cand_count2;    // candidates found by the rescan
+  uint32_t t2;             // the rescan's threshold
+  uint32_t prefix;
   uint32_t kstar;          // the k-th largest key
   uint32_t small_done;     // the one-CTA select did this call (the grid kernel then returns)
-  uint64_t k_rem;          // rank still to find below the prefix
-  uint64_t count_gt;       // elements with key above the prefix range
   uint64_t m;              // K*-ties to keep (lowest indices first)
 };
 
 struct Layout {
-  uint64_t ctl, hs, hc, h0, h1, h2, zero_end, tiles, cand_idx, cand_val, tloc, boff, seg, pj, total;
+  uint64_t state, ctl, hs, hc, hc2, h0, h1, h2, zero_end, tiles, tiles2, cand_idx, cand_val, cand2_idx,
+      cand2_val, tloc, boff, seg, pj, total;
   uint32_t num_tiles, cap;
 };
 
@@ -57,16 +86,21 @@ Layout layout(uint64_t n, uint64_t k) {
   uint64_t cap = 8 * k + 65536;
   L.cap = (uint32_t)(cap < n ? cap : n);
   uint64_t o = 0;
+  L.state = o;    o += align256(sizeof(State));
   L.ctl = o;      o += align256(sizeof(Ctl));
-  L.hs = o;       o += align256(4u * bins(0));
-  L.hc = o;       o += align256(4u * bins(0));   // candidates' first digit (stream pass)
+  L.hs = o;       o += align256(4u * bins(0));   // sample (recovery)
+  L.hc = o;       o += align256(4u * bins(0));   // first-pass candidates' first digit
+  L.hc2 = o;      o += align256(4u * bins(0));   // rescan candidates' first digit
   L.h0 = o;       o += align256(4u * bins(0));
   L.h1 = o;       o += align256(4u * bins(1));
   L.h2 = o;       o += align256(4u * bins(2));
   L.zero_end = o;
   L.tiles = o;    o += align256(8ull * L.num_tiles);
+  L.tiles2 = o;   o += align256(8ull * L.num_tiles);
   L.cand_idx = o; o += align256(4ull * L.cap);
   L.cand_val = o; o += align256(4ull * L.cap);
+  L.cand2_idx = o; o += align256(4ull * L.cap);
+  L.cand2_val = o; o += align256(4ull * L.cap);
   L.tloc = o;     o += align256(8ull * L.num_tiles);   // per-tile (gt, eq) counts, then their scan
   L.boff = o;     o += align256(8ull * 3 * kMaxSelectBlocks);
   L.seg = o;      o += align256(16ull * L.num_tiles);  // small select: P at each tile's segment ends
@@ -90,6 +124,47 @@ template <bool BF16>
 __device__ __forceinline__ float load_g1(const void* g, uint64_t i) {
   if constexpr (BF16) return __uint_as_float(((uint32_t) static_cast<const uint16_t*>(g)[i]) << 16);
   else return static_cast<const float*>(g)[i];
+}
+
+// ---- threshold state ------------------------------------------------------------------------
+__device__ __forceinline__ bool state_valid(const State* st, const StateKey& sk) {
+  return st->magic == kStateMagic && st->n == sk.n && st->k == sk.k && st->resid == sk.resid &&
+         st->tag == sk.tag;
+}
+// The first pass's threshold: K*_prev lowered by delta (in magnitude); "no candidates" when cold.
+__device__ __forceinline__ uint32_t pass1_threshold(const State* st, const StateKey& sk, uint32_t force_t) {
+  if (force_t != kNoForce) return force_t;                 // test hook
+  if (!state_valid(st, sk)) return 0xFFFFFFFFu;           // cold: every key is below it
+  const uint32_t K = st->kstar;
+  if (K >= 0x7F800000u) return 0x7F800000u;               // non-finite k-th key: keep them all
+  const float t = __uint_as_float(K) * (1.0f - st->delta);
+  return __float_as_uint(t) & 0x7FFFFFFFu;
+}
+// After the select (one thread): counters, and the margin controller on the first pass's
+// candidate count: fewer than k -> widen, above the capacity -> narrow, else aim at 1.2-3 k.
+__device__ void state_update(State* st, const StateKey& sk, uint64_t k, uint32_t cap, uint32_t cc,
+                             uint32_t path, uint32_t kstar, uint64_t nonfinite) {
+  const bool warm = state_valid(st, sk);
+  if (!warm) {
+    st->magic = kStateMagic; st->n = sk.n; st->k = sk.k; st->resid = sk.resid; st->tag = sk.tag;
+    st->delta = kDeltaInit;
+    st->calls = st->rescans = st->fallbacks = st->nonfinite_calls = 0;
+  } else {
+    float d = st->delta;
+    if (cc < k) d = d * 2.0f;
+    else if (cc > cap) d = d * 0.5f;
+    else if ((double)cc > 3.0 * (double)k) d = d * 0.75f;
+    else if ((double)cc < 1.2 * (double)k) d = d * 1.5f;
+    st->delta = d < kDeltaMin ? kDeltaMin : (d > kDeltaMax ? kDeltaMax : d);
+  }
+  st->calls += 1;
+  st->rescans += path == 2;
+  st->fallbacks += path == 1;
+  st->nonfinite_calls += nonfinite > 0;
+  st->last_nonfinite = nonfinite;
+  st->kstar = kstar;
+  st->last_cand = cc;
+  st->last_path = path;
 }
 
 // ---- histogram "find": the bin holding the need-th largest key (1-based) --------------------
@@ -126,52 +201,46 @@ __device__ int find_bin_desc(const uint32_t* h, uint64_t need, uint64_t* above_o
   return s_bin;
 }
 
-// ---- K1a: stratified sample of keys -> threshold estimate ----------------------------------
-// Samples are 8-element (32-byte, sector-aligned) micro-chunks spread evenly over [0, n) with a
-// per-call phase, so small parameter segments are represented in proportion (coarse contiguous
-// chunks over-/under-represent segments smaller than their spacing, which biased the tail).
-// Exhaustive mode (small n) visits every micro-chunk.
-// This thread's share of the sample: micro-chunks m = first, first + step, ... -> histogram sh.
-template <bool BF16>
-__device__ __forceinline__ void sample_accumulate(const void* g, const float* r, uint64_t n, uint32_t num_micro,
-                                                  double stride, double phase, int exhaustive, uint32_t* sh,
-                                                  uint32_t first, uint32_t step) {
+// ---- stratified sample of keys (recovery) ---------------------------------------------------
+// Runs after the streaming pass, which stored r = a = g + r for every element it did not record
+// (recorded candidates hold their as-if-selected residual: a bias of < k keys), so the sample
+// reads the residual alone. Samples are 8-element (32-byte, sector-aligned) micro-chunks spread
+// evenly over [0, n) with a per-call phase, so small parameter segments are represented in
+// proportion. Exhaustive mode (small n) visits every micro-chunk. This thread's share:
+// micro-chunks first, first + step, ...
+__device__ __forceinline__ void sample_accumulate(const float* r, uint64_t n, uint32_t num_micro, double stride,
+                                                  double phase, int exhaustive, uint32_t* sh, uint32_t first,
+                                                  uint32_t step) {
   const uint64_t n8 = n / 8;
   for (uint32_t m = first; m < num_micro; m += step) {
     uint64_t c8 = exhaustive ? m : (uint64_t)(((double)m + phase) * stride);
     if (!exhaustive && c8 >= n8) c8 = n8 ? n8 - 1 : 0;
     const uint64_t i = c8 * 8;
     if (i + 8 <= n) {
-      float a[8];
-      const float4 r0 = *reinterpret_cast<const float4*>(r + i);
-      const float4 r1 = *reinterpret_cast<const float4*>(r + i + 4);
-      const float4 g0 = load_g4<BF16>(g, i);
-      const float4 g1 = load_g4<BF16>(g, i + 4);
-      a[0] = g0.x + r0.x; a[1] = g0.y + r0.y; a[2] = g0.z + r0.z; a[3] = g0.w + r0.w;
-      a[4] = g1.x + r1.x; a[5] = g1.y + r1.y; a[6] = g1.z + r1.z; a[7] = g1.w + r1.w;
+      const float4 r0 = __ldcg(reinterpret_cast<const float4*>(r + i));
+      const float4 r1 = __ldcg(reinterpret_cast<const float4*>(r + i + 4));
+      const float a[8] = {r0.x, r0.y, r0.z, r0.w, r1.x, r1.y, r1.z, r1.w};
 #pragma unroll
       for (int e = 0; e < 8; ++e) atomicAdd(&sh[mag_key(a[e]) >> shift(0)], 1u);
     } else {
-      for (uint64_t j = i; j < n; ++j) atomicAdd(&sh[mag_key(load_g1<BF16>(g, j) + r[j]) >> shift(0)], 1u);
+      for (uint64_t j = i; j < n; ++j) atomicAdd(&sh[mag_key(__ldcg(r + j)) >> shift(0)], 1u);
     }
   }
 }
 
-// The threshold from the finished sample histogram hs (block-wide; every thread gets it).
-// Need: exhaustive -> exactly k (threshold = the bin's lower edge: exact, >= k candidates);
-// sampled -> 1.3 x the expected sample count above the k-th key (+8): the candidates land at
-// ~1.3 k, >7 sigma above k for S >= 512 n / k. Within the 12.5 %-wide bin the threshold is
-// placed by an exponential-density model fitted to this bin and the next one up (the tail
-// density falls steeply, so a uniform model lands too high), then moved 10 % toward the lower
-// edge as a safety margin.
+// A threshold from the finished sample histogram hs (block-wide; every thread gets it).
+// Exhaustive -> the lower edge of the bin holding the need_exact-th largest key (exact);
+// sampled -> `factor` x the expected sample count above the k-th key (+8), placed inside its
+// 6 %-wide bin by an exponential-density model of this bin and the next one up, moved 20 %
+// toward the lower edge as a safety margin.
 __device__ __forceinline__ uint32_t threshold_from_sample(const uint32_t* hs, uint64_t n, uint64_t k,
-                                                          uint32_t num_micro, int exhaustive, uint32_t force_t,
-                                                          uint64_t* s_scan) {
+                                                          uint64_t need_exact, double factor, uint32_t num_micro,
+                                                          int exhaustive, uint64_t* s_scan) {
   __shared__ uint32_t s_t;
-  uint64_t S = exhaustive ? n : (uint64_t)num_micro * 8;
-  uint64_t need = exhaustive ? k : (uint64_t)(1.3 * (double)k * (double)S / (double)n) + 8;
+  const uint64_t S = exhaustive ? n : (uint64_t)num_micro * 8;
+  const uint64_t need = exhaustive ? need_exact : (uint64_t)(factor * (double)k * (double)S / (double)n) + 8;
   uint64_t above;
-  int b = find_bin_desc<bins(0)>(hs, need, &above, s_scan);
+  const int b = find_bin_desc<bins(0)>(hs, need, &above, s_scan);
   if (threadIdx.x == 0) {
     uint32_t t = (b < 0) ? 0u : ((uint32_t)b << shift(0));
     if (b >= 0 && !exhaustive) {
@@ -186,61 +255,22 @@ __device__ __forceinline__ uint32_t threshold_from_sample(const uint32_t* hs, ui
         const double el = exp(-lam);
         x = -log(f * (1.0 - el) + el) / lam;
       }
-      x = 0.9 * (x < 0 ? 0 : (x > 1 ? 1 : x));
+      x = 0.8 * (x < 0 ? 0 : (x > 1 ? 1 : x));
       uint32_t off = (uint32_t)(x * (double)(1u << shift(0)));
       if (off >= (1u << shift(0))) off = (1u << shift(0)) - 1;
       t += off;
     }
-    s_t = (force_t != 0xFFFFFFFFu) ? force_t : t;   // force_t: test hook
+    s_t = t;
   }
   __syncthreads();
   return s_t;
 }
 
-template <bool BF16>
-__global__ void __launch_bounds__(kThreads) sample_kernel(const void* g, const float* r, uint64_t n,
-                                                          uint64_t k, uint32_t num_micro, double stride,
-                                                          double phase, int exhaustive, Ctl* ctl,
-                                                          uint32_t* hs, uint32_t force_t) {
-  __shared__ uint32_t sh[bins(0)];
-  __shared__ uint64_t s_scan[kThreads / 32];
-  __shared__ bool s_last;
-  for (int b = threadIdx.x; b < bins(0); b += kThreads) sh[b] = 0;
-  __syncthreads();
-  sample_accumulate<BF16>(g, r, n, num_micro, stride, phase, exhaustive, sh, blockIdx.x * kThreads + threadIdx.x,
-                          gridDim.x * kThreads);
-  __syncthreads();
-  for (int b = threadIdx.x; b < bins(0); b += kThreads)
-    if (sh[b]) atomicAdd(hs + b, sh[b]);
-  __threadfence();
-  __syncthreads();
-  if (threadIdx.x == 0) s_last = (atomicAdd(&ctl->sample_ticket, 1u) == gridDim.x - 1);
-  __syncthreads();
-  if (!s_last) return;
-  __threadfence();
-  const uint32_t t = threshold_from_sample(hs, n, k, num_micro, exhaustive, force_t, s_scan);
-  if (threadIdx.x == 0) {
-    ctl->t_est = t;
-    ctl->k_rem = k;
-  }
-}
-
-// Arguments of the sample when it runs inside the stream kernel (FUSED): one cooperative launch
-// samples, meets at a grid barrier, derives the threshold in every CTA and streams.
-struct SampleArgs {
-  uint64_t k;
-  uint32_t num_micro;
-  double stride, phase;
-  int exhaustive;
-  uint32_t* hs;
-  uint32_t force_t;
-};
-
-// End of a streaming tile (both stream kernels): the tile's candidates go to the buffer (if it has
-// room) and the residual is stored. A candidate that was recorded is stored as if it were selected
-// (r = 0, or a - fp32(bf16(a)) for bf16 values, reading #8): the select kernel then writes r = a
-// back only for the candidates it rejects (~0.3 k), instead of scattering the k selected ones
-// (a scattered 4-byte store costs a 32-byte DRAM read-modify-write).
+// End of a streaming tile: the tile's candidates go to the buffer (if it has room) and the
+// residual is stored. A candidate that was recorded is stored as if it were selected (r = 0, or
+// a - fp32(bf16(a)) for bf16 values, reading #8): the select kernel then writes r = a back only
+// for the candidates it rejects (~0.3 k), instead of scattering the k selected ones (a scattered
+// 4-byte store costs a 32-byte DRAM read-modify-write).
 __device__ __forceinline__ float selected_residual(float a, int vbf16) {
   return vbf16 ? a - __bfloat162float(__float2bfloat16_rn(a)) : 0.0f;
 }
@@ -281,8 +311,38 @@ __device__ __forceinline__ void tile_tail(float (&a)[4][4], uint32_t flags, uint
   }
 }
 
-// ---- K1b: the fused streaming pass ----------------------------------------------------------
-template <bool BF16, bool FUSED = false>
+// Order-preserving compaction of one 4096-element tile: one block scan of 4 x 16-bit per-vector
+// counts. Returns the tile total; vec_base / excl locate this thread's flagged elements.
+__device__ __forceinline__ uint32_t tile_scan(uint32_t flags, uint64_t* s_scan_par, uint32_t (&vec_base)[4],
+                                              uint64_t& excl) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint64_t packed = 0;
+#pragma unroll
+  for (int c = 0; c < 4; ++c) packed |= (uint64_t)__popc((flags >> (4 * c)) & 0xFu) << (16 * c);
+  uint64_t incl = packed;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint64_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+    if (lane >= o) incl += y;
+  }
+  if (lane == 31) s_scan_par[warp] = incl;
+  __syncthreads();
+  uint64_t warp_off = 0, tot = 0;
+#pragma unroll
+  for (int w = 0; w < kThreads / 32; ++w) {
+    uint64_t t = s_scan_par[w];
+    warp_off += (w < warp) ? t : 0;
+    tot += t;
+  }
+  excl = warp_off + incl - packed;
+  uint32_t total = 0;
+#pragma unroll
+  for (int c = 0; c < 4; ++c) { vec_base[c] = total; total += (uint32_t)((tot >> (16 * c)) & 0xFFFF); }
+  return total;
+}
+
+// ---- K1: the fused streaming pass -----------------------------------------------------------
+template <bool BF16>
 __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict__ g,
                                                           float* __restrict__ r, uint64_t n,
                                                           uint32_t num_tiles, Ctl* ctl,
@@ -290,30 +350,14 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
                                                           uint32_t* __restrict__ cand_idx,
                                                           float* __restrict__ cand_val, uint32_t cap,
                                                           int vbf16, uint32_t* __restrict__ hc,
-                                                          SampleArgs sa) {
+                                                          const State* st, StateKey sk, uint32_t force_t) {
   __shared__ uint64_t s_scan[2][kThreads / 32];
   __shared__ uint32_t s_base[2];
   __shared__ uint32_t s_h[bins(0)];               // first-digit histogram of this CTA's candidates
   for (int j = threadIdx.x; j < bins(0); j += kThreads) s_h[j] = 0;
-  uint32_t T;
-  if constexpr (FUSED) {                           // the sample, then a grid barrier, then T
-    __syncthreads();
-    sample_accumulate<BF16>(g, r, n, sa.num_micro, sa.stride, sa.phase, sa.exhaustive, s_h,
-                            blockIdx.x * kThreads + threadIdx.x, gridDim.x * kThreads);
-    __syncthreads();
-    for (int j = threadIdx.x; j < bins(0); j += kThreads)
-      if (s_h[j]) { atomicAdd(sa.hs + j, s_h[j]); s_h[j] = 0; }
-    cg::this_grid().sync();
-    T = threshold_from_sample(sa.hs, n, sa.k, sa.num_micro, sa.exhaustive, sa.force_t, s_scan[0]);
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-      ctl->t_est = T;
-      ctl->k_rem = sa.k;
-    }
-    __syncthreads();
-  } else {
-    T = ctl->t_est;
-  }
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t T = pass1_threshold(st, sk, force_t);
+  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t_est = T;
+  const int tid = threadIdx.x;
   int par = 0;
   for (uint32_t tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, par ^= 1) {
     const uint64_t base = (uint64_t)tile * kTile;
@@ -354,29 +398,9 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
         for (int e = 0; e < 4; ++e)
           if ((flags >> (c * 4 + e)) & 1u) atomicAdd(&s_h[mag_key(a[c][e]) >> shift(0)], 1u);
     }
-    // Order-preserving compaction: one block scan of 4 x 16-bit per-vector counts.
-    uint64_t packed = 0;
-#pragma unroll
-    for (int c = 0; c < 4; ++c) packed |= (uint64_t)__popc((flags >> (4 * c)) & 0xFu) << (16 * c);
-    uint64_t incl = packed;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      uint64_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
-      if (lane >= o) incl += y;
-    }
-    if (lane == 31) s_scan[par][warp] = incl;
-    __syncthreads();
-    uint64_t warp_off = 0, tot = 0;
-#pragma unroll
-    for (int w = 0; w < kThreads / 32; ++w) {
-      uint64_t t = s_scan[par][w];
-      warp_off += (w < warp) ? t : 0;
-      tot += t;
-    }
-    const uint64_t excl = warp_off + incl - packed;
-    uint32_t vec_base[4], total = 0;
-#pragma unroll
-    for (int c = 0; c < 4; ++c) { vec_base[c] = total; total += (uint32_t)((tot >> (16 * c)) & 0xFFFF); }
+    uint32_t vec_base[4];
+    uint64_t excl;
+    const uint32_t total = tile_scan(flags, s_scan[par], vec_base, excl);
     if (tid == 0) {
       uint32_t b = total ? atomicAdd(&ctl->cand_count, total) : 0u;
       s_base[par] = b;
@@ -391,11 +415,11 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
     if (s_h[j]) atomicAdd(hc + j, s_h[j]);
 }
 
-// ---- K1b': the streaming pass with 1-D TMA bulk copies -------------------------------------
+// ---- K1': the streaming pass with 1-D TMA bulk copies (LOWDIFF_STREAM_TMA=1; measured, not the
+// default: DESIGN.md §5) -----------------------------------------------------------------------
 // Same per-tile work as stream_kernel, but the g and r tiles of this CTA's next kStages tiles are
 // in flight as cp.async.bulk copies (one elected thread, completion on an mbarrier per stage)
-// while the current tile is scanned, so the loads never wait behind the block scan's barriers.
-// Full tiles only; the ragged last tile (if any) takes the direct-load path.
+// while the current tile is scanned. Full tiles only; the ragged last tile takes direct loads.
 #ifndef LOWDIFF_STREAM_STAGES
 #define LOWDIFF_STREAM_STAGES 2
 #endif
@@ -407,22 +431,24 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
                                                               uint2* __restrict__ tile_info,
                                                               uint32_t* __restrict__ cand_idx,
                                                               float* __restrict__ cand_val, uint32_t cap,
-                                                              int vbf16, uint32_t* __restrict__ hc) {
-  __shared__ uint32_t s_h[bins(0)];               // first-digit histogram of this CTA's candidates
+                                                              int vbf16, uint32_t* __restrict__ hc,
+                                                              const State* st, StateKey sk, uint32_t force_t) {
+  __shared__ uint32_t s_h[bins(0)];
   for (int j = threadIdx.x; j < bins(0); j += kThreads) s_h[j] = 0;
   constexpr uint32_t kGB = kTile * (BF16 ? 2 : 4), kRB = kTile * 4, kSB = kGB + kRB;
   extern __shared__ __align__(128) uint8_t s_tiles[];          // kStages x {g tile, r tile}
   __shared__ __align__(8) uint64_t s_bar[kStages];
   __shared__ uint64_t s_scan[2][kThreads / 32];
   __shared__ uint32_t s_base[2];
-  const uint32_t T = ctl->t_est;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t T = pass1_threshold(st, sk, force_t);
+  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t_est = T;
+  const int tid = threadIdx.x;
   const uint32_t full_tiles = (uint32_t)(n / kTile);
   auto issue = [&](uint32_t it) {                              // this CTA's it-th tile -> its stage
     const uint32_t tile = blockIdx.x + it * gridDim.x;
     if (tile >= full_tiles) return;
-    const uint32_t st = it % kStages, bar = smem_u32(&s_bar[st]);
-    const uint32_t dst = smem_u32(s_tiles + st * kSB);
+    const uint32_t stg = it % kStages, bar = smem_u32(&s_bar[stg]);
+    const uint32_t dst = smem_u32(s_tiles + stg * kSB);
     mbar_expect_tx(bar, kSB);
     bulk_g2s(dst, static_cast<const uint8_t*>(g) + (uint64_t)tile * kGB, kGB, bar);
     bulk_g2s(dst + kGB, reinterpret_cast<const uint8_t*>(r) + (uint64_t)tile * kRB, kRB, bar);
@@ -440,9 +466,9 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
     float a[4][4];
     uint32_t flags = 0;
     if (tile < full_tiles) {
-      const uint32_t st = it % kStages;
-      mbar_wait(smem_u32(&s_bar[st]), (it / kStages) & 1u);
-      const uint8_t* sg = s_tiles + st * kSB;
+      const uint32_t stg = it % kStages;
+      mbar_wait(smem_u32(&s_bar[stg]), (it / kStages) & 1u);
+      const uint8_t* sg = s_tiles + stg * kSB;
       const float* sr = reinterpret_cast<const float*>(sg + kGB);
 #pragma unroll
       for (int c = 0; c < 4; ++c) {
@@ -474,41 +500,19 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
       for (int e = 0; e < 4; ++e)
         if (tile < full_tiles || i + e < n) flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
     }
-    if (flags) {                                   // the select's first digit, for free
+    if (flags) {
 #pragma unroll
       for (int c = 0; c < 4; ++c)
 #pragma unroll
         for (int e = 0; e < 4; ++e)
           if ((flags >> (c * 4 + e)) & 1u) atomicAdd(&s_h[mag_key(a[c][e]) >> shift(0)], 1u);
     }
-    // Order-preserving compaction: one block scan of 4 x 16-bit per-vector counts.
-    uint64_t packed = 0;
-#pragma unroll
-    for (int c = 0; c < 4; ++c) packed |= (uint64_t)__popc((flags >> (4 * c)) & 0xFu) << (16 * c);
-    uint64_t incl = packed;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      uint64_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
-      if (lane >= o) incl += y;
-    }
-    if (lane == 31) s_scan[par][warp] = incl;
-    __syncthreads();                                  // every thread is done reading this stage
+    uint32_t vec_base[4];
+    uint64_t excl;
+    const uint32_t total = tile_scan(flags, s_scan[par], vec_base, excl);   // every thread is done with the stage
     if (tid == 0) {
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       issue(it + kStages);                            // refill the stage just consumed
-    }
-    uint64_t warp_off = 0, tot = 0;
-#pragma unroll
-    for (int w = 0; w < kThreads / 32; ++w) {
-      uint64_t t = s_scan[par][w];
-      warp_off += (w < warp) ? t : 0;
-      tot += t;
-    }
-    const uint64_t excl = warp_off + incl - packed;
-    uint32_t vec_base[4], total = 0;
-#pragma unroll
-    for (int c = 0; c < 4; ++c) { vec_base[c] = total; total += (uint32_t)((tot >> (16 * c)) & 0xFFFF); }
-    if (tid == 0) {
       uint32_t b = total ? atomicAdd(&ctl->cand_count, total) : 0u;
       s_base[par] = b;
       tile_info[tile] = make_uint2(b, total);
@@ -522,7 +526,26 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
     if (s_h[j]) atomicAdd(hc + j, s_h[j]);
 }
 
-// ---- K1c: exact radix select over the candidates (or the full array) ------------------------
+// ---- K2: exact radix select over the candidates (or the full array) ------------------------
+struct SelArgs {
+  float* r;
+  uint64_t n, k;
+  Ctl* ctl;
+  State* st;
+  StateKey sk;
+  const uint32_t* cidx1; const float* cval1; const uint2* tinfo1;   // first pass
+  uint32_t* cidx2; float* cval2; uint2* tinfo2;                     // rescan
+  uint32_t num_tiles, cap;
+  uint32_t *hs, *hc, *hc2, *h0, *h1, *h2;
+  uint64_t* tloc;
+  uint64_t* boff;
+  uint8_t* pairs;
+  uint32_t num_micro;       // recovery sample
+  double stride, phase;
+  int exhaustive;
+  uint32_t force_t2;        // test hook: the rescan's threshold
+};
+
 // One cooperative launch runs the three digit passes (12 + 10 + 9 bits of the 31-bit key) with a
 // grid barrier after each histogram; every CTA then redoes the tiny 'find' on the L2-resident
 // histogram itself, so no second barrier or serial tail is needed per pass.
@@ -616,50 +639,210 @@ __device__ __forceinline__ uint64_t block_offset(const uint64_t* bsum, uint64_t*
   return tot;
 }
 
+// Put a = g + r back into the residual for every recorded candidate of a buffer (the pass that
+// recorded them stored r as if they were selected). Grid-stride over tiles.
+__device__ __forceinline__ void restore_recorded(float* r, const uint2* tinfo, const uint32_t* cidx,
+                                                 const float* cval, uint32_t num_tiles, uint32_t cap) {
+  const uint64_t stride = (uint64_t)gridDim.x * kThreads;
+  for (uint64_t t = (uint64_t)blockIdx.x * kThreads + threadIdx.x; t < num_tiles; t += stride) {
+    const uint2 ti = tinfo[t];
+    if (ti.y && (uint64_t)ti.x + ti.y <= cap)
+      for (uint32_t j = 0; j < ti.y; ++j) r[cidx[ti.x + j]] = cval[ti.x + j];
+  }
+}
+
+// Recovery rescan: rebuild the candidate set at threshold T2 from the residual, with the first
+// pass's recorded candidates overlaid from its buffer (their r holds the as-if-selected value).
+// Writes the rescan buffer, its tile table and first-digit histogram, and fixes r wherever an
+// element's recorded state changes (recorded now, not before: as-if-selected; before, not now: a).
+__device__ void rescan(const SelArgs& A, uint32_t T2, int vbf16, float* s_ov, uint32_t* s_bits, uint32_t* s_h,
+                       uint64_t (*s_scan)[kThreads / 32], uint32_t* s_base) {
+  const int tid = threadIdx.x;
+  const uint64_t n = A.n;
+  for (int j = tid; j < bins(0); j += kThreads) s_h[j] = 0;
+  __syncthreads();
+  int par = 0;
+  for (uint32_t tile = blockIdx.x; tile < A.num_tiles; tile += gridDim.x, par ^= 1) {
+    const uint64_t base = (uint64_t)tile * kTile;
+    const bool full = base + kTile <= n;
+    float a[4][4];
+    if (full) {
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        const float4 v = __ldcg(reinterpret_cast<const float4*>(A.r + base + c * 1024 + tid * 4));
+        a[c][0] = v.x; a[c][1] = v.y; a[c][2] = v.z; a[c][3] = v.w;
+      }
+    } else {
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const uint64_t i = base + c * 1024 + tid * 4 + e;
+          a[c][e] = i < n ? A.r[i] : 0.f;
+        }
+    }
+    const uint2 s1 = A.tinfo1[tile];
+    uint32_t old = 0;
+    if (s1.y && (uint64_t)s1.x + s1.y <= A.cap) {       // block-uniform
+      if (tid < kTile / 32) s_bits[tid] = 0;
+      __syncthreads();
+      for (uint32_t j = tid; j < s1.y; j += kThreads) {
+        const uint32_t o = A.cidx1[s1.x + j] - (uint32_t)base;
+        s_ov[o] = A.cval1[s1.x + j];
+        atomicOr(&s_bits[o >> 5], 1u << (o & 31));
+      }
+      __syncthreads();
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const uint32_t o = c * 1024 + tid * 4 + e;
+          if ((s_bits[o >> 5] >> (o & 31)) & 1u) { a[c][e] = s_ov[o]; old |= 1u << (c * 4 + e); }
+        }
+    }
+    uint32_t flags = 0;
+#pragma unroll
+    for (int c = 0; c < 4; ++c)
+#pragma unroll
+      for (int e = 0; e < 4; ++e)
+        if (full || base + c * 1024 + tid * 4 + e < n) flags |= (mag_key(a[c][e]) >= T2 ? 1u : 0u) << (c * 4 + e);
+    if (flags) {
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          if ((flags >> (c * 4 + e)) & 1u) atomicAdd(&s_h[mag_key(a[c][e]) >> shift(0)], 1u);
+    }
+    uint32_t vec_base[4];
+    uint64_t excl;
+    const uint32_t total = tile_scan(flags, s_scan[par], vec_base, excl);
+    if (tid == 0) {
+      const uint32_t b = total ? atomicAdd(&A.ctl->cand_count2, total) : 0u;
+      s_base[par] = b;
+      A.tinfo2[tile] = make_uint2(b, total);
+    }
+    __syncthreads();
+    const uint32_t b = s_base[par];
+    const bool rec = total && (uint64_t)b + total <= A.cap;
+    if (rec && flags) {
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        uint32_t pos = b + vec_base[c] + (uint32_t)((excl >> (16 * c)) & 0xFFFF);
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          if (flags & (1u << (c * 4 + e))) {
+            A.cidx2[pos] = (uint32_t)(base + c * 1024 + tid * 4 + e);
+            A.cval2[pos] = a[c][e];
+            ++pos;
+          }
+      }
+    }
+    const uint32_t sel = rec ? flags : 0u;
+    uint32_t diff = sel ^ old;
+    while (diff) {
+      const int bit = __ffs(diff) - 1;
+      diff &= diff - 1;
+      const int c = bit >> 2, e = bit & 3;
+      const float v = a[c][e];
+      A.r[base + c * 1024 + tid * 4 + e] = ((sel >> bit) & 1u) ? selected_residual(v, vbf16) : v;
+    }
+  }
+  __syncthreads();
+  for (int j = tid; j < bins(0); j += kThreads)
+    if (s_h[j]) atomicAdd(A.hc2 + j, s_h[j]);
+}
+
 template <bool VBF16>
-__global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__ r, uint64_t n, uint64_t k,
-                                                          Ctl* ctl, const float* __restrict__ cand_val,
-                                                          const uint32_t* __restrict__ cand_idx,
-                                                          const uint2* __restrict__ tile_info,
-                                                          uint32_t num_tiles, uint32_t cap, uint32_t* h0,
-                                                          uint32_t* h1, uint32_t* h2, uint32_t* hc,
-                                                          uint64_t* tloc, uint64_t* boff, uint8_t* pairs) {
+__global__ void __launch_bounds__(kThreads, 4) select_kernel(SelArgs A) {
   cg::grid_group grid = cg::this_grid();
   __shared__ uint32_t sh[bins(0)];
-  __shared__ uint64_t s_scan[kThreads / 32];
+  __shared__ uint64_t s_scan[2][kThreads / 32];
+  Ctl* ctl = A.ctl;
   if (ctl->small_done) return;                     // the one-CTA select did this call (uniform)
+  const uint64_t n = A.n, k = A.k;
+  const uint32_t cap = A.cap, num_tiles = A.num_tiles;
   const uint32_t cc = ctl->cand_count;
-  const uint32_t mode = (cc >= k && cc <= cap) ? 0u : 1u;
-  const float* src = mode ? r : cand_val;
-  const uint64_t N = mode ? n : (uint64_t)cc;
-  if (mode) {
-    // full-array fallback: the stream pass stored the recorded candidates' residual as if they
-    // were selected; put a = g + r back for them first (their values are in the buffer)
-    const uint64_t stride = (uint64_t)gridDim.x * kThreads;
-    for (uint64_t t = (uint64_t)blockIdx.x * kThreads + threadIdx.x; t < num_tiles; t += stride) {
-      const uint2 ti = tile_info[t];
-      if (ti.y && (uint64_t)ti.x + ti.y <= cap)
-        for (uint32_t j = 0; j < ti.y; ++j) r[cand_idx[ti.x + j]] = cand_val[ti.x + j];
+  // the candidate set the select runs on: the first pass's, unless it missed
+  const uint32_t* cidx = A.cidx1;
+  const float* cval = A.cval1;
+  const uint2* tinfo = A.tinfo1;
+  const uint32_t* hfirst = A.hc;
+  uint64_t N = cc;
+  uint32_t mode = 0;
+  if (cc < k || cc > cap) {                        // recovery (uniform)
+    __shared__ float s_ov[kTile];
+    __shared__ uint32_t s_bits[kTile / 32];
+    __shared__ uint32_t s_base[2];
+    __shared__ uint32_t s_t2;
+    const uint32_t T = ctl->t_est;
+    bool try_rescan = true;
+    if (cc > cap) {
+      // too many: the k-th key's bin in the exact first-digit histogram of ALL candidates
+      uint64_t above;
+      const int bk = find_bin_desc<bins(0)>(A.hc, k, &above, s_scan[0]);
+      const uint32_t lo_edge = bk < 0 ? 0u : (uint32_t)bk << shift(0);
+      const uint64_t cnt = bk < 0 ? ~0ull : above + __ldcg(A.hc + bk);
+      if (threadIdx.x == 0) s_t2 = lo_edge > T ? lo_edge : T;
+      try_rescan = cnt <= cap;
+    } else {
+      // too few: a stratified sample of the keys (the first pass's candidates read as their
+      // as-if-selected residual: a bias of < k keys, covered by the 2x margin; exhaustive
+      // sampling asks for the k - cc still missing instead)
+      for (int j = threadIdx.x; j < bins(0); j += kThreads) sh[j] = 0;
+      __syncthreads();
+      sample_accumulate(A.r, n, A.num_micro, A.stride, A.phase, A.exhaustive, sh,
+                        blockIdx.x * kThreads + threadIdx.x, gridDim.x * kThreads);
+      __syncthreads();
+      for (int j = threadIdx.x; j < bins(0); j += kThreads)
+        if (sh[j]) atomicAdd(A.hs + j, sh[j]);
+      grid.sync();
+      uint32_t t2 = threshold_from_sample(A.hs, n, k, k - cc, 2.0, A.num_micro, A.exhaustive, s_scan[0]);
+      if (t2 >= T) t2 = __float_as_uint(__uint_as_float(T) * 0.875f) & 0x7FFFFFFFu;
+      if (threadIdx.x == 0) s_t2 = t2;
     }
-    grid.sync();
+    __syncthreads();
+    uint32_t T2 = s_t2;
+    if (A.force_t2 != kNoForce) T2 = A.force_t2;   // test hook
+    if (try_rescan) {
+      rescan(A, T2, VBF16 ? 1 : 0, s_ov, s_bits, sh, s_scan, s_base);
+      grid.sync();
+      const uint32_t cc2 = __ldcg(&ctl->cand_count2);
+      if (cc2 >= k && cc2 <= cap) {
+        cidx = A.cidx2; cval = A.cval2; tinfo = A.tinfo2; hfirst = A.hc2; N = cc2; mode = 2;
+      } else {
+        restore_recorded(A.r, A.tinfo2, A.cidx2, A.cval2, num_tiles, cap);
+        mode = 1;
+      }
+    } else {
+      restore_recorded(A.r, A.tinfo1, A.cidx1, A.cval1, num_tiles, cap);
+      mode = 1;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t2 = T2;
+    if (mode == 1) { N = n; grid.sync(); }
   }
+  const float* src = mode == 1 ? A.r : cval;
   uint32_t prefix = 0;
   uint64_t need = k;
-  // candidate mode: the stream pass already histogrammed the candidates' first digit (hc)
-  select_pass<0>(src, N, sh, mode ? h0 : hc, prefix, need, s_scan, grid, mode != 0);
-  select_pass<1>(src, N, sh, h1, prefix, need, s_scan, grid);
-  select_pass<2>(src, N, sh, h2, prefix, need, s_scan, grid);
+  // candidate modes: the pass that built the set already histogrammed its first digit
+  select_pass<0>(src, N, sh, mode == 1 ? A.h0 : const_cast<uint32_t*>(hfirst), prefix, need, s_scan[0], grid,
+                 mode == 1);
+  select_pass<1>(src, N, sh, A.h1, prefix, need, s_scan[0], grid);
+  select_pass<2>(src, N, sh, A.h2, prefix, need, s_scan[0], grid);
   const uint32_t K = prefix;
   const uint64_t m = need;                         // K*-ties to keep (lowest indices first)
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     ctl->mode = mode;
     ctl->kstar = K;
     ctl->m = m;
+    const uint32_t* hf = mode == 1 ? A.h0 : hfirst;
+    uint64_t nonfinite = 0;                        // keys >= +Inf: all of them are candidates
+    for (uint32_t b = kNonFiniteBin; b < (uint32_t)bins(0); ++b) nonfinite += __ldcg(hf + b);
+    state_update(A.st, A.sk, k, cap, cc, mode, K, nonfinite);
   }
   // ---- fused ordered emission ----
-  // A streaming tile's candidates sit contiguously in the buffer, in index order (candidate mode),
-  // or the tile is its own 4096 residual elements (full mode, the fallback). A group of g lanes
-  // (a power of two covering the mean segment length, 4..32) owns one tile at a time:
+  // A streaming tile's candidates sit contiguously in the buffer, in index order (candidate modes),
+  // or the tile is its own 4096 residual elements (full mode). A group of g lanes (a power of two
+  // covering the mean segment length, 4..32) owns one tile at a time:
   //  (A) per tile: (count > K*, count == K*) over its segment -> tcnt[t]
   //  (B) exclusive scan of tcnt over tiles (block chunks + block offsets)
   //  (C) per tile again: ballot prefixes inside the segment give each kept candidate its slot
@@ -669,9 +852,10 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
   while (((uint64_t)G << ts_log) < num_tiles) ++ts_log;
   uint32_t glog = 2;
   while (glog < 5 && ((uint64_t)num_tiles << glog) < N) ++glog;
-  const float* vsrc = mode ? r : cand_val;
+  float* r = A.r;
+  const float* vsrc = mode == 1 ? r : cval;
   auto segment = [&](uint64_t t) -> uint2 {      // (first buffer position, length) of tile t
-    if (mode == 0) return tile_info[t];
+    if (mode != 1) return tinfo[t];
     const uint64_t b0 = t * kTile;
     return make_uint2((uint32_t)b0, (uint32_t)((n - b0) < (uint64_t)kTile ? n - b0 : kTile));
   };
@@ -680,7 +864,8 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
   const uint64_t tpw = 32u >> glog;                // tiles per warp per round
   const uint64_t wstride = (uint64_t)G * (kThreads / 32) * tpw;
   const uint64_t tfirst = (((uint64_t)b * kThreads + threadIdx.x) >> 5) * tpw + (lane >> glog);
-  uint64_t* tcnt = tloc;
+  uint64_t* tcnt = A.tloc;
+  uint64_t* boff = A.boff;
   // (A)
   for (uint64_t tw = tfirst - (lane >> glog); tw < num_tiles; tw += wstride) {   // warp-uniform
     const uint64_t t = tw + (lane >> glog);
@@ -701,14 +886,15 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
   grid.sync();
   // (B)
   const uint64_t t0 = (uint64_t)b << ts_log, t1 = (t0 + (1ull << ts_log) < num_tiles) ? t0 + (1ull << ts_log) : num_tiles;
-  const uint64_t ttot = t0 < t1 ? chunk_scan(t0, t1, [&](uint64_t t) { return tcnt[t]; }, tcnt, s_scan) : 0;
+  const uint64_t ttot = t0 < t1 ? chunk_scan(t0, t1, [&](uint64_t t) { return tcnt[t]; }, tcnt, s_scan[0]) : 0;
   if (threadIdx.x == 0) boff[b] = ttot;
   grid.sync();
-  const uint64_t toff = block_offset(boff, s_scan);
+  const uint64_t toff = block_offset(boff, s_scan[0]);
   __syncthreads();
   if (threadIdx.x == 0) boff[G + b] = toff;
   grid.sync();
   // (C)
+  uint8_t* pairs = A.pairs;
   uint32_t* out_idx = reinterpret_cast<uint32_t*>(pairs);
   uint8_t* out_val = pairs + pad16(4 * k);
   if (b == 0 && threadIdx.x < 16) {                // zero the 16-byte padding of both sections
@@ -720,7 +906,7 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
   const uint32_t lt = (1u << gl) - 1;
   // the next round's tile (segment, prefix) is loaded while the current one is emitted, and the
   // group's loads of two iterations are issued together: the loop is load-latency bound
-  auto tinfo = [&](uint64_t tw, uint2& ti, uint64_t& tp) {
+  auto tinfo_at = [&](uint64_t tw, uint2& ti, uint64_t& tp) {
     const uint64_t t = tw + (lane >> glog);
     const bool tv = t < num_tiles;
     ti = tv ? segment(t) : make_uint2(0u, 0u);
@@ -729,11 +915,11 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
   uint64_t tw = tfirst - (lane >> glog);
   uint2 ti = make_uint2(0u, 0u);
   uint64_t tp = 0;
-  if (tw < num_tiles) tinfo(tw, ti, tp);
+  if (tw < num_tiles) tinfo_at(tw, ti, tp);
   for (; tw < num_tiles; tw += wstride) {          // warp-uniform
     uint2 nti = make_uint2(0u, 0u);
     uint64_t ntp = 0;
-    if (tw + wstride < num_tiles) tinfo(tw + wstride, nti, ntp);
+    if (tw + wstride < num_tiles) tinfo_at(tw + wstride, nti, ntp);
     uint64_t gtb = tp >> 32, eqb = tp & 0xFFFFFFFFull;
     const uint32_t len_max = __reduce_max_sync(0xFFFFFFFFu, ti.y);
     for (uint32_t j0 = 0; j0 < len_max; j0 += 2 * g) {
@@ -745,7 +931,7 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
         const uint32_t j = j0 + h * g + gl;
         in2[h] = j < ti.y;
         a2[h] = in2[h] ? vsrc[(uint64_t)ti.x + j] : 0.f;
-        id2[h] = in2[h] ? (mode ? ti.x + j : cand_idx[(uint64_t)ti.x + j]) : 0u;
+        id2[h] = in2[h] ? (mode == 1 ? ti.x + j : cidx[(uint64_t)ti.x + j]) : 0u;
       }
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
@@ -764,12 +950,12 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
           if constexpr (VBF16) {
             const __nv_bfloat16 hb = __float2bfloat16_rn(a);
             reinterpret_cast<__nv_bfloat16*>(out_val)[pos] = hb;
-            if (mode) r[idx] = a - __bfloat162float(hb);   // exact (Sterbenz), reading #8
+            if (mode == 1) r[idx] = a - __bfloat162float(hb);   // exact (Sterbenz), reading #8
           } else {
             reinterpret_cast<float*>(out_val)[pos] = a;
-            if (mode) r[idx] = 0.0f;
+            if (mode == 1) r[idx] = 0.0f;
           }
-        } else if (in && !mode) {
+        } else if (in && mode != 1) {
           r[idx] = a;                              // a rejected candidate keeps all of a
         }
         gtb += __popc(bg);
@@ -782,7 +968,7 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(float* __restrict__
 }
 
 
-// ---- K1c': small problems (<= 2^15 candidates): the same select + ordered emission in ONE CTA ----
+// ---- K2': small problems (<= 2^15 candidates): the same select + ordered emission in ONE CTA ----
 // The grid kernel's ~10 dependent phases each pay a grid barrier; for a few thousand candidates
 // (C1) one CTA does every phase behind __syncthreads. Work is split by candidate-buffer position:
 //   digits : shared-memory histograms of the candidates (12 bits from the stream pass, 10, 9)
@@ -857,7 +1043,7 @@ select_small_kernel(float* __restrict__ r, uint64_t k, Ctl* ctl, const float* __
                     const uint32_t* __restrict__ cand_idx, const uint2* __restrict__ tile_info,
                     uint32_t num_tiles, uint32_t cap, const uint32_t* __restrict__ hc,
                     uint64_t* __restrict__ toff, ulonglong2* __restrict__ seg, uint64_t* __restrict__ pj,
-                    uint8_t* __restrict__ pairs) {
+                    uint8_t* __restrict__ pairs, State* st, StateKey sk) {
   const uint32_t cc = ctl->cand_count;
   if (!(cc >= k && cc <= cap && cc <= kSmallMaxCand)) return;   // the grid kernel does this call
   __shared__ uint32_t s_h0[bins(0)], s_h1[bins(1)], s_h2[bins(2)];
@@ -893,7 +1079,12 @@ select_small_kernel(float* __restrict__ r, uint64_t k, Ctl* ctl, const float* __
   need -= above;
   const uint32_t K = (p1 << 9) | d2;
   const uint64_t m = need;                         // K*-ties to keep (lowest indices first)
-  if (tid == 0) { ctl->mode = 0; ctl->kstar = K; ctl->m = m; ctl->small_done = 1; }
+  if (tid == 0) {
+    ctl->mode = 0; ctl->kstar = K; ctl->m = m; ctl->small_done = 1;
+    uint64_t nonfinite = 0;
+    for (uint32_t b = kNonFiniteBin; b < (uint32_t)bins(0); ++b) nonfinite += s_h0[b];
+    state_update(st, sk, k, cap, cc, 0, K, nonfinite);
+  }
   auto flag = [&](uint32_t j) -> uint64_t {        // packed (key > K*, key == K*) of position j
     const uint32_t key = mag_key(cand_val[j]);
     return ((uint64_t)(key > K) << 32) | (uint64_t)(key == K);
@@ -983,7 +1174,18 @@ select_small_kernel(float* __restrict__ r, uint64_t k, Ctl* ctl, const float* __
 }
 
 int g_stream_blocks_f32 = 0, g_stream_blocks_bf16 = 0;
-uint32_t g_force_t = 0xFFFFFFFFu;       // test hook: override the sampled threshold
+uint32_t g_force_t = kNoForce;          // test hooks: override the first-pass / rescan thresholds
+uint32_t g_force_t2 = kNoForce;
+
+int device_sms() {
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms < 1) sms = kNumSMs;
+  }
+  return sms;
+}
 
 int g_tma_blocks_f32 = 0, g_tma_blocks_bf16 = 0;
 int stream_tma_smem(bool bf16) { return kStages * kTile * ((bf16 ? 2 : 4) + 4); }
@@ -999,7 +1201,7 @@ int stream_tma_blocks(bool bf16) {
       cudaFuncSetAttribute(stream_tma_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, stream_tma_kernel<false>, kThreads, smem);
     }
-    cache = (per_sm > 0 ? per_sm : 1) * kNumSMs;
+    cache = (per_sm > 0 ? per_sm : 1) * device_sms();
   }
   return cache;
 }
@@ -1010,27 +1212,62 @@ int stream_blocks(bool bf16) {
     int per_sm = 0;
     if (bf16) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, stream_kernel<true>, kThreads, 0);
     else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, stream_kernel<false>, kThreads, 0);
-    int dev = 0, sms = kNumSMs;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cache = (per_sm > 0 ? per_sm : 4) * sms;
+    cache = (per_sm > 0 ? per_sm : 4) * device_sms();
   }
   return cache;
+}
+
+const void* select_fn(bool vbf) {
+  return vbf ? (const void*)select_kernel<true> : (const void*)select_kernel<false>;
+}
+
+// CTAs per SM the cooperative select may use: its occupancy limit over all four variants
+int select_max_per_sm() {
+  static int sel_max = 0;
+  if (!sel_max) {
+    sel_max = kMaxSelectBlocks;
+    for (int q = 0; q < 2; ++q) {
+      int a = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, select_fn(q), kThreads, 0);
+      if (a < sel_max) sel_max = a;
+    }
+    if (sel_max < 1) sel_max = 1;
+    const int cap = kMaxSelectBlocks / device_sms();
+    if (sel_max > (cap < 1 ? 1 : cap)) sel_max = cap < 1 ? 1 : cap;
+  }
+  return sel_max;
 }
 
 }  // namespace
 
 uint64_t compress_ws_bytes(uint64_t n, uint64_t k) { return layout(n, k).total; }
 
-void compress_force_threshold(int enable, uint32_t key) { g_force_t = enable ? key : 0xFFFFFFFFu; }
+void compress_force_threshold(int which, int enable, uint32_t key) {
+  (which == 0 ? g_force_t : g_force_t2) = enable ? key : kNoForce;
+}
 
 lowdiff_status compress_stats(const void* ws, uint64_t n, uint64_t k, uint64_t out[6], cudaStream_t s) {
-  (void)n; (void)k;
+  const Layout L = layout(n, k);
   Ctl c;
-  LD_CUDA(cudaMemcpyAsync(&c, ws, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "stats copy");
+  LD_CUDA(cudaMemcpyAsync(&c, static_cast<const uint8_t*>(ws) + L.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s),
+          "stats copy");
   LD_CUDA(cudaStreamSynchronize(s), "stats sync");
   out[0] = c.t_est; out[1] = c.cand_count; out[2] = c.mode; out[3] = c.kstar; out[4] = c.m;
-  out[5] = layout(n, k).cap;
+  out[5] = L.cap;
+  return LOWDIFF_OK;
+}
+
+lowdiff_status compress_counters(const void* ws, cudaStream_t s, uint64_t out[8]) {
+  State st;
+  LD_CUDA(cudaMemcpyAsync(&st, ws, sizeof(State), cudaMemcpyDeviceToHost, s), "counters copy");
+  LD_CUDA(cudaStreamSynchronize(s), "counters sync");
+  if (st.magic != kStateMagic) {
+    for (int i = 0; i < 8; ++i) out[i] = 0;
+    return LOWDIFF_OK;
+  }
+  out[0] = st.calls; out[1] = st.rescans; out[2] = st.fallbacks; out[3] = st.nonfinite_calls;
+  out[4] = st.last_nonfinite; out[5] = st.last_cand; out[6] = st.kstar;
+  out[7] = (uint64_t)((double)st.delta * 4294967296.0);     // delta in 2^-32 units
   return LOWDIFF_OK;
 }
 
@@ -1039,10 +1276,12 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   const Layout L = layout(n, k);
   uint8_t* w = static_cast<uint8_t*>(ws);
   Ctl* ctl = reinterpret_cast<Ctl*>(w + L.ctl);
-  LD_CUDA(cudaMemsetAsync(w, 0, L.zero_end, s), "memset compress workspace");
+  State* st = reinterpret_cast<State*>(w + L.state);
+  LD_CUDA(cudaMemsetAsync(w + L.ctl, 0, L.zero_end - L.ctl, s), "memset compress workspace");
+  const StateKey sk{n, k, (uint64_t)(uintptr_t)residual, (uint64_t)(gdt | (vdt << 8))};
 
-  // sample size: >= 512 expected keys above the k-th (S >= 512 n / k: the 1.3x target, ~666
-  // sampled keys, is then ~7.5 sigma of the count above k), >= 64 Ki, power of 2
+  // recovery sample size: >= 512 expected keys above the k-th (S >= 512 n / k: the 2x target is
+  // then > 10 sigma of the count above k), >= 64 Ki, power of 2; every micro-chunk when S >= n/2
   uint64_t S = 65536;
   while ((double)S * (double)k < 512.0 * (double)n && S < (1ull << 26)) S <<= 1;
   const int exhaustive = (S >= n / 2) ? 1 : 0;
@@ -1050,32 +1289,10 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   const double stride = exhaustive ? 1.0 : (double)(n / 8) / (double)micro;
   static uint64_t calls = 0;                       // per-call phase (golden-ratio sequence)
   const double phase = exhaustive ? 0.0 : (double)((++calls * 0x9E3779B97F4A7C15ull) >> 11) * 0x1p-53;
-  uint64_t sg = (micro + kThreads - 1) / kThreads;
-  if (sg > 2ull * kNumSMs) sg = 2ull * kNumSMs;
-  const int sample_grid = (int)sg;
-  uint32_t* hs = reinterpret_cast<uint32_t*>(w + L.hs);
-  static int use_tma = -1, fuse_sample = -1;
+  static int use_tma = -1;
   if (use_tma < 0) {
     const char* e = getenv("LOWDIFF_STREAM_TMA");
     use_tma = e ? atoi(e) : 0;
-    e = getenv("LOWDIFF_FUSED_SAMPLE");           // 0 never, 1 always, 2 (default) small grids
-    fuse_sample = e ? atoi(e) : 2;
-  }
-  // fused: the sample runs at the start of the (then cooperative) stream kernel, behind one grid
-  // barrier, instead of as its own launch that ends in a one-CTA threshold step. Measured: it pays
-  // off when the stream grid is small (every tile in one wave: n <= resident CTAs x 4096, C1:
-  // compress 0.161 -> 0.130 ms per 8 calls); with the full 740-CTA grid (C2, C3) the barrier and
-  // the per-CTA threshold step cost as much as the separate launch.
-  const bool fused = !use_tma && (fuse_sample == 1 ||
-                                  (fuse_sample == 2 && L.num_tiles <= (uint32_t)stream_blocks(gdt == LOWDIFF_BF16)));
-  SampleArgs sa{k, micro, stride, phase, exhaustive, hs, g_force_t};
-  if (!fused) {
-    if (gdt == LOWDIFF_BF16)
-      LD_LAUNCH("compress_sample", s, sample_kernel<true>, sample_grid, kThreads, 0, grad, residual, n,
-                k, micro, stride, phase, exhaustive, ctl, hs, g_force_t);
-    else
-      LD_LAUNCH("compress_sample", s, sample_kernel<false>, sample_grid, kThreads, 0, grad, residual,
-                n, k, micro, stride, phase, exhaustive, ctl, hs, g_force_t);
   }
 
   uint2* tiles = reinterpret_cast<uint2*>(w + L.tiles);
@@ -1090,85 +1307,72 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
     const int smem = stream_tma_smem(bf);
     if (bf)
       LD_LAUNCH("compress_stream", s, stream_tma_kernel<true>, grid, kThreads, smem, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, st, sk, g_force_t);
     else
       LD_LAUNCH("compress_stream", s, stream_tma_kernel<false>, grid, kThreads, smem, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, st, sk, g_force_t);
   } else {
     int grid = stream_blocks(bf);
     if ((uint32_t)grid > L.num_tiles) grid = (int)L.num_tiles;
-    if (fused) {                                   // co-resident by construction (occupancy grid)
-      uint32_t nt = L.num_tiles, cp = L.cap;
-      void* args[] = {(void*)&grad, (void*)&residual, (void*)&n, (void*)&nt, (void*)&ctl, (void*)&tiles,
-                      (void*)&cidx, (void*)&cval, (void*)&cp, (void*)&vbf, (void*)&hcand, (void*)&sa};
-      ProfScope prof("compress_stream", s);
-      const void* fn = bf ? (const void*)stream_kernel<true, true> : (const void*)stream_kernel<false, true>;
-      LD_CUDA(cudaLaunchCooperativeKernel(fn, grid, kThreads, args, 0, s), "stream launch");
-      note_launch();
-    } else if (bf) {
+    if (bf)
       LD_LAUNCH("compress_stream", s, stream_kernel<true>, grid, kThreads, 0, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, sa);
-    } else {
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, st, sk, g_force_t);
+    else
       LD_LAUNCH("compress_stream", s, stream_kernel<false>, grid, kThreads, 0, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, sa);
-    }
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, st, sk, g_force_t);
   }
 
-  {
-    static int sel_max = 0;                        // occupancy limit (CTAs per SM), both variants
-    if (!sel_max) {
-      int a = 0, b2 = 0;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, select_kernel<false>, kThreads, 0);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b2, select_kernel<true>, kThreads, 0);
-      sel_max = a < b2 ? a : b2;
-      if (sel_max < 1) sel_max = 1;
-      if (sel_max > kMaxSelectBlocks / kNumSMs) sel_max = kMaxSelectBlocks / kNumSMs;
-    }
-    // CTAs per SM: more hide the latency of the emission loop at large k, fewer make the grid
-    // syncs and histogram flushes cheaper at small k (measured, profiles/README.md).
-    int want = k >= (1u << 18) ? 4 : 2;
-    if (const char* e = getenv("LOWDIFF_SELECT_PER_SM")) want = atoi(e);
-    if (want < 1) want = 1;
-    if (want > sel_max) want = sel_max;
-    int sel_grid = want * kNumSMs;
-    if (const char* e = getenv("LOWDIFF_SELECT_GRID")) {   // experiments: explicit CTA count
-      const int gq = atoi(e);
-      if (gq >= 1 && gq <= sel_max * kNumSMs && gq <= kMaxSelectBlocks) sel_grid = gq;
-    }
-    float* rr = residual;
-    uint32_t *h0 = reinterpret_cast<uint32_t*>(w + L.h0), *h1 = reinterpret_cast<uint32_t*>(w + L.h1),
-             *h2 = reinterpret_cast<uint32_t*>(w + L.h2);
-    uint64_t* tloc = reinterpret_cast<uint64_t*>(w + L.tloc);
-    uint64_t* boff = reinterpret_cast<uint64_t*>(w + L.boff);
-    uint8_t* pp = static_cast<uint8_t*>(pairs);
-    const uint32_t* cidx_c = cidx;
-    const uint2* tiles_c = tiles;
-    uint32_t cap = L.cap, nt = L.num_tiles;
-    void* args[] = {(void*)&rr, (void*)&n, (void*)&k, (void*)&ctl, (void*)&cval, (void*)&cidx_c,
-                    (void*)&tiles_c, (void*)&nt, (void*)&cap, (void*)&h0, (void*)&h1, (void*)&h2,
-                    (void*)&hcand, (void*)&tloc, (void*)&boff, (void*)&pp};
-    ProfScope prof("compress_select", s);
-    static int use_small = -1;
-    if (use_small < 0) {
-      const char* e = getenv("LOWDIFF_SELECT_SMALL");
-      use_small = e ? atoi(e) : 1;
-    }
-    if (use_small && 4 * k <= kSmallMaxCand) {   // a few thousand candidates: one CTA does it all
-      ulonglong2* seg = reinterpret_cast<ulonglong2*>(w + L.seg);
-      uint64_t* pj = reinterpret_cast<uint64_t*>(w + L.pj);
-      if (vdt == LOWDIFF_BF16)
-        select_small_kernel<true><<<1, kSmallThreads, 0, s>>>(rr, k, ctl, cval, cidx, tiles, nt, cap, hcand, tloc,
-                                                               seg, pj, pp);
-      else
-        select_small_kernel<false><<<1, kSmallThreads, 0, s>>>(rr, k, ctl, cval, cidx, tiles, nt, cap, hcand, tloc,
-                                                                seg, pj, pp);
-      note_launch();
-    }
-    const void* fn = vdt == LOWDIFF_BF16 ? (const void*)select_kernel<true> : (const void*)select_kernel<false>;
-    LD_CUDA(cudaLaunchCooperativeKernel(fn, sel_grid, kThreads, args, 0, s), "select launch");
+  const int sel_max = select_max_per_sm();
+  // CTAs per SM: more hide the latency of the emission loop at large k, fewer make the grid
+  // syncs and histogram flushes cheaper at small k (measured, profiles/README.md).
+  int want = k >= (1u << 18) ? 4 : 2;
+  if (const char* e = getenv("LOWDIFF_SELECT_PER_SM")) want = atoi(e);
+  if (want < 1) want = 1;
+  if (want > sel_max) want = sel_max;
+  int sel_grid = want * device_sms();
+  if (sel_grid > kMaxSelectBlocks) sel_grid = kMaxSelectBlocks;
+  if (const char* e = getenv("LOWDIFF_SELECT_GRID")) {   // experiments: explicit CTA count
+    const int gq = atoi(e);
+    if (gq >= 1 && gq <= sel_max * device_sms() && gq <= kMaxSelectBlocks) sel_grid = gq;
+  }
+  SelArgs A;
+  A.r = residual; A.n = n; A.k = k; A.ctl = ctl; A.st = st; A.sk = sk;
+  A.cidx1 = cidx; A.cval1 = cval; A.tinfo1 = tiles;
+  A.cidx2 = reinterpret_cast<uint32_t*>(w + L.cand2_idx);
+  A.cval2 = reinterpret_cast<float*>(w + L.cand2_val);
+  A.tinfo2 = reinterpret_cast<uint2*>(w + L.tiles2);
+  A.num_tiles = L.num_tiles; A.cap = L.cap;
+  A.hs = reinterpret_cast<uint32_t*>(w + L.hs);
+  A.hc = hcand;
+  A.hc2 = reinterpret_cast<uint32_t*>(w + L.hc2);
+  A.h0 = reinterpret_cast<uint32_t*>(w + L.h0);
+  A.h1 = reinterpret_cast<uint32_t*>(w + L.h1);
+  A.h2 = reinterpret_cast<uint32_t*>(w + L.h2);
+  A.tloc = reinterpret_cast<uint64_t*>(w + L.tloc);
+  A.boff = reinterpret_cast<uint64_t*>(w + L.boff);
+  A.pairs = static_cast<uint8_t*>(pairs);
+  A.num_micro = micro; A.stride = stride; A.phase = phase; A.exhaustive = exhaustive;
+  A.force_t2 = g_force_t2;
+  ProfScope prof("compress_select", s);
+  static int use_small = -1;
+  if (use_small < 0) {
+    const char* e = getenv("LOWDIFF_SELECT_SMALL");
+    use_small = e ? atoi(e) : 1;
+  }
+  if (use_small && 4 * k <= kSmallMaxCand) {   // a few thousand candidates: one CTA does it all
+    ulonglong2* seg = reinterpret_cast<ulonglong2*>(w + L.seg);
+    uint64_t* pj = reinterpret_cast<uint64_t*>(w + L.pj);
+    if (vbf)
+      select_small_kernel<true><<<1, kSmallThreads, 0, s>>>(residual, k, ctl, cval, cidx, tiles, L.num_tiles, L.cap,
+                                                             hcand, A.tloc, seg, pj, A.pairs, st, sk);
+    else
+      select_small_kernel<false><<<1, kSmallThreads, 0, s>>>(residual, k, ctl, cval, cidx, tiles, L.num_tiles, L.cap,
+                                                              hcand, A.tloc, seg, pj, A.pairs, st, sk);
     note_launch();
   }
-
+  void* args[] = {(void*)&A};
+  LD_CUDA(cudaLaunchCooperativeKernel(select_fn(vbf), sel_grid, kThreads, args, 0, s), "select launch");
+  note_launch();
   return cuda_status(cudaGetLastError(), "compress launch");
 }
 

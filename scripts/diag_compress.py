@@ -19,6 +19,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", type=int, default=3)
 ap.add_argument("--iters", type=int, default=300)
 ap.add_argument("--cycle", type=int, default=16)
+ap.add_argument("--every", type=int, default=16)
 a = ap.parse_args()
 cfg = CONFIGS[a.config]
 dev = torch.device("cuda", 0)
@@ -30,7 +31,12 @@ for it in range(a.iters):
     ld.compress(grads[it % a.cycle], r, cfg.k, vdt=cfg.vdt)
     st = ld.compress_stats(cfg.n, cfg.k)
     fallbacks += st["fallback"]
-    if it < 20 or it % 16 == 0 or st["fallback"]:
+    rescans = locals().get("rescans", 0) + st["rescan"]
+    if it < 20 or it % a.every == 0 or st["path"]:
+        import struct
+        f = lambda key: struct.unpack("<f", struct.pack("<I", int(key)))[0]
         print(f"it {it:4d} cand/k {st['candidates'] / cfg.k:7.3f} cap/k {st['capacity'] / cfg.k:6.2f} "
-              f"fallback {st['fallback']} t_est {st['t_est']:#x} kstar {st['kstar']:#x}", flush=True)
-print(f"fallbacks: {fallbacks} / {a.iters}")
+              f"path {st['path']} t_est {f(st['t_est']):.6g} kstar {f(st['kstar']):.6g} "
+              f"ratio {f(st['t_est']) / max(f(st['kstar']), 1e-30):.4f}", flush=True)
+print(f"fallbacks: {fallbacks} rescans: {rescans} / {a.iters}")
+print(ld.compress_counters(cfg.n, cfg.k))
