@@ -382,7 +382,8 @@ def run_ours(args, cfg):
     cc2 = ld.compress_counters(ws=cws)
     # compress paths over both passes: 0 = warm first-pass candidates, 2 = rescan
     # recovery inside the select, 1 = exact full-array select; counted on the device
-    paths = {"calls": cc2["calls"] - cc0["calls"], "rescans": cc2["rescans"] - cc0["rescans"],
+    paths = {"calls": cc2["calls"] - cc0["calls"], "fast_select": cc2["fast_calls"] - cc0["fast_calls"],
+             "rescans": cc2["rescans"] - cc0["rescans"],
              "fallbacks": cc2["fallbacks"] - cc0["fallbacks"],
              "timed": {q: cc1[q] - cc0[q] for q in ("calls", "rescans", "fallbacks")},
              "since_start": {q: cc2[q] for q in ("calls", "rescans", "fallbacks", "nonfinite_calls")},

@@ -75,6 +75,38 @@ uint64_t lowdiff_pairs_bytes(uint64_t k, lowdiff_dtype vdt);
 lowdiff_status lowdiff_shard_bounds(uint64_t n, int32_t nranks, int32_t rank, uint64_t* lo, uint64_t* hi);
 
 /* ---------------------------------------------------------------------------------------------
+ * (0) Plan — the paper's problem statement: a flat gradient of n elements compressed at ratio rho
+ *     (P:130), differentials batched B per write (batching size b) and a
+ *     full checkpoint every full_every iterations (f = 1/FCF), on rank `rank` of
+ *     `nranks` data-parallel ranks.
+ *   lowdiff_plan_init fills k = lowdiff_k_for_density(n, rho) and the rank's shard [lo, hi)
+ *     (lowdiff_shard_bounds). Errors: EINVAL (n = 0 or n >= 2^31, rho not in (0, 1], B = 0 or
+ *     B > 255, nranks < 1, rank out of range, unknown dtype).
+ *   lowdiff_plan_record_due(t): the record-boundary policy for iteration t (0-based; DESIGN.md
+ *     reading #25). A full checkpoint C^F_t (M_t, before G~_t is applied) is due before iteration
+ *     t when t % full_every == 0 (full_every = 0: only at t = 0). A record never spans a full
+ *     checkpoint: the open record closes after iteration t when it holds B iterations, or when the
+ *     next iteration starts with a full checkpoint — then it is a SHORT record (B' < B iterations;
+ *     legal, the header carries B'). Outputs (host, any may be NULL): *full_checkpoint_due,
+ *     *close_record, *batch_len = iterations in the open record including t (= B' when it closes).
+ *     What a failure loses: iterations after the last closed and persisted record.
+ * ------------------------------------------------------------------------------------------- */
+typedef struct {
+  uint64_t n;
+  double rho;
+  uint64_t k;
+  uint32_t B;
+  uint32_t full_every;      /* FCF in iterations; 0 = only the initial full checkpoint */
+  int32_t gdt, vdt;         /* lowdiff_dtype of the gradient and of the emitted values */
+  int32_t nranks, rank;
+  uint64_t lo, hi;
+} lowdiff_plan;
+lowdiff_status lowdiff_plan_init(lowdiff_plan* plan, uint64_t n, double rho, uint32_t B, uint32_t full_every,
+                                 lowdiff_dtype gdt, lowdiff_dtype vdt, int32_t nranks, int32_t rank);
+lowdiff_status lowdiff_plan_record_due(const lowdiff_plan* plan, uint64_t t, int32_t* close_record,
+                                       uint32_t* batch_len, int32_t* full_checkpoint_due);
+
+/* ---------------------------------------------------------------------------------------------
  * (1) Compress — Comp(G_{i,t}), Alg.1 line 4; "sparsification" at ratio rho.
  *     Exact top-k with error feedback (north_star; readings #1-#8):
  *       a = fp32(grad) + residual                         (one fp32 add; bf16 widening exact)
@@ -253,8 +285,9 @@ lowdiff_status lowdiff_stage_d2h(const void* d_record, uint64_t bytes, void* h_p
  *     step with gradient 0 at absent indices (Comp^{-1}): SGD (x -= lr*(g + wd x)),
  *     SGD-momentum (torch.optim.SGD conventions), Adam (Eq.1; bias-corrected, eps
  *     after the sqrt). STACK records: one step per iteration (lr = lr[j]). SUM records: one step
- *     with the summed gradient and lr[0] — exact trajectory only for SGD, so momentum/Adam
- *     need allow_accumulated_sum (else EUNSUPPORTED); a SUM record's lr[] must be constant.
+ *     with the summed gradient and lr[0] — exact trajectory only for plain SGD (weight decay 0),
+ *     so momentum, Adam and SGD with weight decay need allow_accumulated_sum (else EUNSUPPORTED;
+ *     reading #13); a SUM record's lr[] must be constant.
  *     Scalars are computed on the host in double and rounded once to fp32.
  *   recs[i].d_record: device record bytes; recs[i].h_head: HOST copy of (at least) its header
  *     and lr[] (e.g. the pinned staging buffer); h_head_len >= 80 + 4B.
@@ -396,17 +429,19 @@ lowdiff_status lowdiff_optimal_config(const lowdiff_config_model* m, double* f_s
  *     "merge_pack", "replay_dense", "replay_sparse", "starts".
  * ------------------------------------------------------------------------------------------- */
 uint64_t       lowdiff_launch_count(void);
-/* After a lowdiff_compress on `stream` with workspace `ws` (syncs the stream): out6 = {first-pass
- * threshold key, first-pass candidates found, path (0 = first-pass candidates, 2 = rescan
- * candidates, 1 = full-array select), k-th key, ties kept, candidate capacity}. Diagnostics. */
+/* After a lowdiff_compress on `stream` with workspace `ws` (syncs the stream): out8 = {first-pass
+ * threshold key, first-pass candidates found, path (3 = first-pass candidates, fast select; 0 =
+ * first-pass candidates, general select; 2 = rescan candidates; 1 = full-array select), k-th key,
+ * ties kept, candidate capacity, fine-histogram shift, candidates in the k-th key's fine bin}. */
 lowdiff_status lowdiff_compress_stats(const void* ws, uint64_t n, uint64_t k, lowdiff_stream_t stream,
-                                      uint64_t* out6);
-/* The threshold state of the residual `ws` was last used with (syncs `stream`): out8 =
+                                      uint64_t* out8);
+/* The threshold state of the residual `ws` was last used with (syncs `stream`): out9 =
  * {calls, rescans (path 2), full-array fallbacks (path 1), calls that saw non-finite a, non-finite
- * count of the last call, first-pass candidates of the last call, last k-th key, margin x 2^32}.
+ * count of the last call, first-pass candidates of the last call, last k-th key, margin x 2^32,
+ * fast-select calls (path 3)}.
  * All zero for a workspace never used by lowdiff_compress. Counters restart when the workspace
  * moves to another residual / n / k. */
-lowdiff_status lowdiff_compress_counters(const void* ws, lowdiff_stream_t stream, uint64_t* out8);
+lowdiff_status lowdiff_compress_counters(const void* ws, lowdiff_stream_t stream, uint64_t* out9);
 /* Test hooks: while enabled, every later lowdiff_compress uses `key` as its first-pass candidate
  * threshold (lowdiff_debug_force_threshold: drives the rescan recovery) or as the rescan's
  * threshold (lowdiff_debug_force_rescan_threshold: drives the exact full-array path). */

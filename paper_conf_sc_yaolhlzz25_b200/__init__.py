@@ -63,6 +63,13 @@ class State(C.Structure):
                 ("x0", C.c_void_p), ("m0", C.c_void_p), ("v0", C.c_void_p)]
 
 
+class Plan(C.Structure):
+    """lowdiff_plan: the problem statement (n, rho -> k, B, FCF, dtypes, rank -> shard)."""
+    _fields_ = [("n", C.c_uint64), ("rho", C.c_double), ("k", C.c_uint64), ("B", C.c_uint32),
+                ("full_every", C.c_uint32), ("gdt", C.c_int32), ("vdt", C.c_int32), ("nranks", C.c_int32),
+                ("rank", C.c_int32), ("lo", C.c_uint64), ("hi", C.c_uint64)]
+
+
 class RecordView(C.Structure):
     _fields_ = [("d_record", C.c_void_p), ("h_head", C.c_void_p), ("h_head_len", C.c_uint64)]
 
@@ -83,7 +90,7 @@ EXPORTS = [
     "lowdiff_update_workspace_size", "lowdiff_update", "lowdiff_dense_update", "lowdiff_host_update",
     "lowdiff_p2p_window_bytes", "lowdiff_p2p_export_handle", "lowdiff_p2p_init", "lowdiff_p2p_init_local",
     "lowdiff_p2p_destroy", "lowdiff_p2p_slot", "lowdiff_p2p_allgather_sparse", "lowdiff_p2p_status",
-    "lowdiff_batch_merge_ex",
+    "lowdiff_batch_merge_ex", "lowdiff_plan_init", "lowdiff_plan_record_due",
 ]
 
 _lib = None
@@ -151,6 +158,8 @@ def lib() -> C.CDLL:
         "lowdiff_p2p_slot": ([vp, vp], vp),
         "lowdiff_p2p_allgather_sparse": ([vp, vp, u64, u64, i32, vp, vp, u64, vp, vp, u64, vp], i32),
         "lowdiff_p2p_status": ([vp], i32),
+        "lowdiff_plan_init": ([vp, u64, f64, C.c_uint32, C.c_uint32, i32, i32, i32, i32], i32),
+        "lowdiff_plan_record_due": ([vp, u64, vp, vp, vp], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -210,6 +219,24 @@ def shard_bounds(n: int, nranks: int, rank: int) -> tuple[int, int]:
     lo, hi = C.c_uint64(), C.c_uint64()
     _check(lib().lowdiff_shard_bounds(n, nranks, rank, C.byref(lo), C.byref(hi)), "shard_bounds")
     return lo.value, hi.value
+
+
+def plan_init(n: int, rho: float, B: int, full_every: int, gdt="f32", vdt="f32", nranks: int = 1,
+              rank: int = 0) -> Plan:
+    """lowdiff_plan_init: k, the rank's shard [lo, hi) and the batching / full-checkpoint policy."""
+    p = Plan()
+    _check(lib().lowdiff_plan_init(C.byref(p), n, float(rho), B, full_every, _DT[gdt], _DT[vdt], nranks, rank),
+           "plan_init")
+    return p
+
+
+def plan_record_due(plan: Plan, t: int) -> tuple[bool, int, bool]:
+    """lowdiff_plan_record_due for iteration t: (close the open record after t, its length so far
+    including t, a full checkpoint is due before t) — DESIGN.md reading #25."""
+    close, blen, full = C.c_int32(), C.c_uint32(), C.c_int32()
+    _check(lib().lowdiff_plan_record_due(C.byref(plan), t, C.byref(close), C.byref(blen), C.byref(full)),
+           "plan_record_due")
+    return bool(close.value), int(blen.value), bool(full.value)
 
 
 class ConfigModel(C.Structure):
@@ -661,14 +688,17 @@ def replay_parallel(state: dict, opt: dict, records, ws=None, stream=None) -> di
 # ---- instrumentation --------------------------------------------------------------------------------
 def compress_stats(n: int, k: int, device="cuda", stream=None, ws=None) -> dict:
     """Diagnostics of the last compress that used `ws` (default: the cached workspace; syncs).
-    path: 0 = first-pass candidates, 2 = rescan recovery, 1 = exact full-array select."""
+    path: 3 = first-pass candidates with the fast select, 0 = first-pass candidates with the general
+    select, 2 = rescan recovery, 1 = exact full-array select."""
     if ws is None:
         ws = workspace(compress_workspace_size(n, k), device, "compress")
-    out = (C.c_uint64 * 6)()
+    out = (C.c_uint64 * 8)()
     _check(lib().lowdiff_compress_stats(_cuda(ws, "ws"), n, k, _stream(stream), out), "compress_stats")
-    d = dict(zip(("t_est", "candidates", "path", "kstar", "ties_kept", "capacity"), list(out)))
+    d = dict(zip(("t_est", "candidates", "path", "kstar", "ties_kept", "capacity", "fine_shift", "inbin"),
+                 list(out)))
     d["fallback"] = int(d["path"] == 1)
     d["rescan"] = int(d["path"] == 2)
+    d["first_pass"] = int(d["path"] in (0, 3))
     return d
 
 
@@ -677,11 +707,12 @@ def compress_counters(n: int = 0, k: int = 0, device="cuda", stream=None, ws=Non
     fallbacks, non-finite calls/count, last candidates, last k-th key, margin."""
     if ws is None:
         ws = workspace(compress_workspace_size(n, k), device, "compress")
-    out = (C.c_uint64 * 8)()
+    out = (C.c_uint64 * 9)()
     _check(lib().lowdiff_compress_counters(_cuda(ws, "ws"), _stream(stream), out), "compress_counters")
     v = list(out)
     return {"calls": v[0], "rescans": v[1], "fallbacks": v[2], "nonfinite_calls": v[3],
-            "last_nonfinite": v[4], "last_candidates": v[5], "kstar": v[6], "delta": v[7] / 2.0 ** 32}
+            "last_nonfinite": v[4], "last_candidates": v[5], "kstar": v[6], "delta": v[7] / 2.0 ** 32,
+            "fast_calls": v[8]}
 
 
 def debug_force_threshold(key: int | None):

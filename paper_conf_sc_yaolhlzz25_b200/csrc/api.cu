@@ -128,6 +128,36 @@ lowdiff_status lowdiff_shard_bounds(uint64_t n, int32_t nranks, int32_t rank, ui
   return LOWDIFF_OK;
 }
 
+// ---- (0) plan: the problem statement and the record-boundary policy (reading #25) -------------
+lowdiff_status lowdiff_plan_init(lowdiff_plan* p, uint64_t n, double rho, uint32_t B, uint32_t full_every,
+                                 lowdiff_dtype gdt, lowdiff_dtype vdt, int32_t nranks, int32_t rank) {
+  if (!p) return fail(LOWDIFF_EINVAL, "plan_init: null plan");
+  if (n == 0 || n >= (1ull << 31)) return fail(LOWDIFF_EINVAL, "plan_init: need 1 <= n < 2^31");
+  if (!(rho > 0.0 && rho <= 1.0)) return fail(LOWDIFF_EINVAL, "plan_init: rho must be in (0, 1]");
+  if (B == 0 || B > 255) return fail(LOWDIFF_EINVAL, "plan_init: need 1 <= B <= 255");
+  if ((gdt != LOWDIFF_F32 && gdt != LOWDIFF_BF16) || (vdt != LOWDIFF_F32 && vdt != LOWDIFF_BF16))
+    return fail(LOWDIFF_EINVAL, "plan_init: bad dtype");
+  uint64_t lo, hi;
+  lowdiff_status s = lowdiff_shard_bounds(n, nranks, rank, &lo, &hi);
+  if (s) return s;
+  p->n = n; p->rho = rho; p->k = lowdiff_k_for_density(n, rho); p->B = B; p->full_every = full_every;
+  p->gdt = gdt; p->vdt = vdt; p->nranks = nranks; p->rank = rank; p->lo = lo; p->hi = hi;
+  return LOWDIFF_OK;
+}
+
+lowdiff_status lowdiff_plan_record_due(const lowdiff_plan* p, uint64_t t, int32_t* close_record,
+                                       uint32_t* batch_len, int32_t* full_checkpoint_due) {
+  if (!p || p->B == 0) return fail(LOWDIFF_EINVAL, "plan_record_due: bad plan");
+  const uint64_t F = p->full_every;
+  const uint64_t f = F ? t / F * F : 0;            // the full checkpoint the open chain starts from
+  const uint64_t pos = (t - f) % p->B;             // t's place in its record
+  const bool full_next = F && (t + 1) % F == 0;    // a full checkpoint is due before t + 1
+  if (full_checkpoint_due) *full_checkpoint_due = (F ? t % F == 0 : t == 0) ? 1 : 0;
+  if (close_record) *close_record = (pos + 1 == p->B || full_next) ? 1 : 0;
+  if (batch_len) *batch_len = (uint32_t)(pos + 1);
+  return LOWDIFF_OK;
+}
+
 // ---- (1) compress ---------------------------------------------------------------------------
 lowdiff_status lowdiff_compress_workspace_size(uint64_t n, uint64_t k, uint64_t* bytes) {
   if (!bytes || n == 0 || n >= (1ull << 31) || k == 0 || k > n)
@@ -393,8 +423,9 @@ static lowdiff_status build_recinfo(const lowdiff_state* st, const lowdiff_opt* 
     t += h.B;
     const float* lr = reinterpret_cast<const float*>(static_cast<const uint8_t*>(recs[q].h_head) + 80);
     if (h.mode == LOWDIFF_MERGE_SUM) {
-      if (o->kind != LOWDIFF_OPT_SGD && !o->allow_accumulated_sum)
-        return fail(LOWDIFF_EUNSUPPORTED, "replay: SUM record with momentum/Adam needs allow_accumulated_sum");
+      if ((o->kind != LOWDIFF_OPT_SGD || o->weight_decay != 0.0) && !o->allow_accumulated_sum)   // reading #13
+        return fail(LOWDIFF_EUNSUPPORTED,
+                    "replay: SUM record with momentum, Adam or weight decay needs allow_accumulated_sum");
       for (uint32_t j = 1; j < h.B; ++j)
         if (memcmp(&lr[j], &lr[0], 4) != 0) return fail(LOWDIFF_EUNSUPPORTED, "replay: SUM record with varying lr");
     }
@@ -568,15 +599,15 @@ lowdiff_status lowdiff_debug_force_rescan_threshold(int32_t enable, uint32_t key
   return LOWDIFF_OK;
 }
 
-lowdiff_status lowdiff_compress_counters(const void* ws, lowdiff_stream_t stream, uint64_t* out8) {
-  if (!ws || !out8) return fail(LOWDIFF_EINVAL, "compress_counters: null");
-  return compress_counters(ws, (cudaStream_t)stream, out8);
+lowdiff_status lowdiff_compress_counters(const void* ws, lowdiff_stream_t stream, uint64_t* out9) {
+  if (!ws || !out9) return fail(LOWDIFF_EINVAL, "compress_counters: null");
+  return compress_counters(ws, (cudaStream_t)stream, out9);
 }
 
 lowdiff_status lowdiff_compress_stats(const void* ws, uint64_t n, uint64_t k, lowdiff_stream_t stream,
-                                      uint64_t* out6) {
-  if (!ws || !out6) return fail(LOWDIFF_EINVAL, "compress_stats: null");
-  return compress_stats(ws, n, k, out6, (cudaStream_t)stream);
+                                      uint64_t* out8) {
+  if (!ws || !out8) return fail(LOWDIFF_EINVAL, "compress_stats: null");
+  return compress_stats(ws, n, k, out8, (cudaStream_t)stream);
 }
 
 lowdiff_status lowdiff_profile_enable(int32_t on) {

@@ -44,7 +44,7 @@ constexpr uint32_t kNoForce = 0xFFFFFFFFu;
 // digit p = (key >> shift(p)) & (bins(p) - 1): 12 + 10 + 9 bits of the 31-bit key
 __host__ __device__ constexpr int bins(int p) { return p == 0 ? 4096 : (p == 1 ? 1024 : 512); }
 __host__ __device__ constexpr int shift(int p) { return p == 0 ? 19 : (p == 1 ? 9 : 0); }
-constexpr uint32_t kNonFiniteBin = 0x7F800000u >> 19;   // first-digit bins >= this hold Inf/NaN keys
+constexpr uint32_t kMaxChunks = 4096;            // fast select: chunks of tiles with a kept count each
 
 // Persistent per-residual state (the first 256 bytes of the workspace; never cleared by a call).
 // It is valid only for the (n, k, residual, dtypes) it was written for; anything else (a fresh or
@@ -54,7 +54,7 @@ struct __align__(256) State {
   uint64_t magic, n, k, resid, tag;
   uint32_t kstar;           // the previous call's exact k-th key
   float delta;              // relative margin below it for the next threshold
-  uint64_t calls, rescans, fallbacks, nonfinite_calls, last_nonfinite;
+  uint64_t calls, rescans, fallbacks, nonfinite_calls, last_nonfinite, fast_calls;
   uint32_t last_cand, last_path;
 };
 struct StateKey {
@@ -64,19 +64,22 @@ constexpr float kDeltaInit = 1.0f / 64, kDeltaMin = 1.0f / 8192, kDeltaMax = 0.5
 
 struct __align__(256) Ctl {
   uint32_t t_est;          // the first pass's threshold: candidates have key >= t_est
-  uint32_t mode;           // path: 0 = first-pass candidates, 2 = rescan candidates, 1 = full array
+  uint32_t mode;           // path: 0/3 = first-pass candidates (3: fast select), 2 = rescan, 1 = full array
   uint32_t cand_count;     // candidates found by the streaming pass (may exceed capacity)
   uint32_t cand_count2;    // candidates found by the rescan
   uint32_t t2;             // the rescan's threshold
   uint32_t prefix;
   uint32_t kstar;          // the k-th largest key
   uint32_t small_done;     // the one-CTA select did this call (the grid kernel then returns)
+  uint32_t fine_shift;     // the first pass's candidate histogram: bin = min((key - t_est) >> fine_shift, 4095)
+  uint32_t nonfinite;      // elements with |a| = Inf or NaN (the streaming pass sees every a)
+  uint32_t inbin_count;    // fast select: candidates in the k-th key's fine bin
   uint64_t m;              // K*-ties to keep (lowest indices first)
 };
 
 struct Layout {
-  uint64_t state, ctl, hs, hc, hc2, h0, h1, h2, zero_end, tiles, tiles2, cand_idx, cand_val, cand2_idx,
-      cand2_val, tloc, boff, seg, pj, total;
+  uint64_t state, ctl, hs, hc, hc2, h0, h1, h2, hl, ctot, zero_end, tiles, tiles2, cand_idx, cand_val, cand2_idx,
+      cand2_val, tloc, tk, bits, inbin, boff, seg, pj, total;
   uint32_t num_tiles, cap;
 };
 
@@ -89,11 +92,13 @@ Layout layout(uint64_t n, uint64_t k) {
   L.state = o;    o += align256(sizeof(State));
   L.ctl = o;      o += align256(sizeof(Ctl));
   L.hs = o;       o += align256(4u * bins(0));   // sample (recovery)
-  L.hc = o;       o += align256(4u * bins(0));   // first-pass candidates' first digit
+  L.hc = o;       o += align256(4u * bins(0));   // first-pass candidates' fine bins (relative to T)
   L.hc2 = o;      o += align256(4u * bins(0));   // rescan candidates' first digit
   L.h0 = o;       o += align256(4u * bins(0));
   L.h1 = o;       o += align256(4u * bins(1));
   L.h2 = o;       o += align256(4u * bins(2));
+  L.hl = o;       o += align256(4u * bins(0));
+  L.ctot = o;     o += align256(8u * kMaxChunks);
   L.zero_end = o;
   L.tiles = o;    o += align256(8ull * L.num_tiles);
   L.tiles2 = o;   o += align256(8ull * L.num_tiles);
@@ -102,6 +107,9 @@ Layout layout(uint64_t n, uint64_t k) {
   L.cand2_idx = o; o += align256(4ull * L.cap);
   L.cand2_val = o; o += align256(4ull * L.cap);
   L.tloc = o;     o += align256(8ull * L.num_tiles);   // per-tile (gt, eq) counts, then their scan
+  L.tk = o;       o += align256(8ull * L.num_tiles);   // fast select: (>, ==) counts per tile
+  L.bits = o;     o += align256(8ull * (L.cap / 32 + 1));   // fast select: (>, ==) bits per position
+  L.inbin = o;    o += align256(8ull * L.cap);         // fast select: the undecided (position, value)
   L.boff = o;     o += align256(8ull * 3 * kMaxSelectBlocks);
   L.seg = o;      o += align256(16ull * L.num_tiles);  // small select: P at each tile's segment ends
   L.pj = o;       o += align256(8ull * (L.cap < kSmallMaxCand ? L.cap : kSmallMaxCand));   // P per position
@@ -140,6 +148,26 @@ __device__ __forceinline__ uint32_t pass1_threshold(const State* st, const State
   const float t = __uint_as_float(K) * (1.0f - st->delta);
   return __float_as_uint(t) & 0x7FFFFFFFu;
 }
+// The first pass's candidate histogram is relative to T: bin = min((key - T) >> s, 4095), with s
+// the smallest shift whose bins 0..4094 reach K*_prev (1 + 2 delta): around the expected k-th key
+// the bins are a few key units wide, so the select finds K* with one pass over the candidates.
+// Cold or forced thresholds use s = 19 (the bins then cover every key >= T).
+__device__ __forceinline__ uint32_t fine_shift(const State* st, const StateKey& sk, uint32_t T, uint32_t force_t) {
+  if (force_t != kNoForce || !state_valid(st, sk)) return 19;
+  const uint32_t K = st->kstar;
+  if (K >= 0x7F800000u || T >= 0x7F800000u) return 19;
+  uint32_t top = __float_as_uint(__uint_as_float(K) * (1.0f + 2.0f * st->delta)) & 0x7FFFFFFFu;
+  if (top >= 0x7F800000u) top = 0x7F7FFFFFu;
+  const uint64_t range = top > T ? top - T : 1;
+  uint32_t sh = 0;
+  while (sh < 19 && (4095ull << sh) < range) ++sh;
+  return sh;
+}
+__device__ __forceinline__ uint32_t fine_bin(uint32_t key, uint32_t T, uint32_t s) {   // key >= T
+  const uint32_t d = (key - T) >> s;
+  return d < 4095u ? d : 4095u;
+}
+
 // After the select (one thread): counters, and the margin controller on the first pass's
 // candidate count: fewer than k -> widen, above the capacity -> narrow, else aim at 1.2-3 k.
 __device__ void state_update(State* st, const StateKey& sk, uint64_t k, uint32_t cap, uint32_t cc,
@@ -148,7 +176,7 @@ __device__ void state_update(State* st, const StateKey& sk, uint64_t k, uint32_t
   if (!warm) {
     st->magic = kStateMagic; st->n = sk.n; st->k = sk.k; st->resid = sk.resid; st->tag = sk.tag;
     st->delta = kDeltaInit;
-    st->calls = st->rescans = st->fallbacks = st->nonfinite_calls = 0;
+    st->calls = st->rescans = st->fallbacks = st->nonfinite_calls = st->fast_calls = 0;
   } else {
     float d = st->delta;
     if (cc < k) d = d * 2.0f;
@@ -160,6 +188,7 @@ __device__ void state_update(State* st, const StateKey& sk, uint64_t k, uint32_t
   st->calls += 1;
   st->rescans += path == 2;
   st->fallbacks += path == 1;
+  st->fast_calls += path == 3;
   st->nonfinite_calls += nonfinite > 0;
   st->last_nonfinite = nonfinite;
   st->kstar = kstar;
@@ -350,14 +379,17 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
                                                           uint32_t* __restrict__ cand_idx,
                                                           float* __restrict__ cand_val, uint32_t cap,
                                                           int vbf16, uint32_t* __restrict__ hc,
+                                                          uint64_t* __restrict__ tk,
                                                           const State* st, StateKey sk, uint32_t force_t) {
   __shared__ uint64_t s_scan[2][kThreads / 32];
   __shared__ uint32_t s_base[2];
-  __shared__ uint32_t s_h[bins(0)];               // first-digit histogram of this CTA's candidates
+  __shared__ uint32_t s_h[bins(0)];               // fine histogram of this CTA's candidates
   for (int j = threadIdx.x; j < bins(0); j += kThreads) s_h[j] = 0;
   const uint32_t T = pass1_threshold(st, sk, force_t);
-  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t_est = T;
+  const uint32_t FS = fine_shift(st, sk, T, force_t);
+  if (blockIdx.x == 0 && threadIdx.x == 0) { ctl->t_est = T; ctl->fine_shift = FS; }
   const int tid = threadIdx.x;
+  uint32_t nonfinite = 0;
   int par = 0;
   for (uint32_t tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, par ^= 1) {
     const uint64_t base = (uint64_t)tile * kTile;
@@ -376,7 +408,10 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
         a[c][0] = gv[c].x + rv[c].x; a[c][1] = gv[c].y + rv[c].y;
         a[c][2] = gv[c].z + rv[c].z; a[c][3] = gv[c].w + rv[c].w;
 #pragma unroll
-        for (int e = 0; e < 4; ++e) flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
+        for (int e = 0; e < 4; ++e) {
+          flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
+          nonfinite += mag_key(a[c][e]) >= 0x7F800000u;
+        }
       }
     } else {
 #pragma unroll
@@ -388,6 +423,7 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
           if (i < n) {
             a[c][e] = load_g1<BF16>(g, i) + r[i];
             flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
+            nonfinite += mag_key(a[c][e]) >= 0x7F800000u;
           }
         }
     }
@@ -396,7 +432,7 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
       for (int c = 0; c < 4; ++c)
 #pragma unroll
         for (int e = 0; e < 4; ++e)
-          if ((flags >> (c * 4 + e)) & 1u) atomicAdd(&s_h[mag_key(a[c][e]) >> shift(0)], 1u);
+          if ((flags >> (c * 4 + e)) & 1u) atomicAdd(&s_h[fine_bin(mag_key(a[c][e]), T, FS)], 1u);
     }
     uint32_t vec_base[4];
     uint64_t excl;
@@ -405,11 +441,13 @@ __global__ void __launch_bounds__(kThreads) stream_kernel(const void* __restrict
       uint32_t b = total ? atomicAdd(&ctl->cand_count, total) : 0u;
       s_base[par] = b;
       tile_info[tile] = make_uint2(b, total);
+      tk[tile] = 0;
     }
     __syncthreads();
     tile_tail(a, flags, total, vec_base, excl, s_base[par], cap, base, n, base + kTile <= n, vbf16, r,
               cand_idx, cand_val);
   }
+  if (nonfinite) atomicAdd(&ctl->nonfinite, nonfinite);
   __syncthreads();
   for (int j = threadIdx.x; j < bins(0); j += kThreads)
     if (s_h[j]) atomicAdd(hc + j, s_h[j]);
@@ -432,6 +470,7 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
                                                               uint32_t* __restrict__ cand_idx,
                                                               float* __restrict__ cand_val, uint32_t cap,
                                                               int vbf16, uint32_t* __restrict__ hc,
+                                                              uint64_t* __restrict__ tk,
                                                               const State* st, StateKey sk, uint32_t force_t) {
   __shared__ uint32_t s_h[bins(0)];
   for (int j = threadIdx.x; j < bins(0); j += kThreads) s_h[j] = 0;
@@ -441,8 +480,10 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
   __shared__ uint64_t s_scan[2][kThreads / 32];
   __shared__ uint32_t s_base[2];
   const uint32_t T = pass1_threshold(st, sk, force_t);
-  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->t_est = T;
+  const uint32_t FS = fine_shift(st, sk, T, force_t);
+  if (blockIdx.x == 0 && threadIdx.x == 0) { ctl->t_est = T; ctl->fine_shift = FS; }
   const int tid = threadIdx.x;
+  uint32_t nonfinite = 0;
   const uint32_t full_tiles = (uint32_t)(n / kTile);
   auto issue = [&](uint32_t it) {                              // this CTA's it-th tile -> its stage
     const uint32_t tile = blockIdx.x + it * gridDim.x;
@@ -498,14 +539,17 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
       const uint64_t i = base + c * 1024 + tid * 4;
 #pragma unroll
       for (int e = 0; e < 4; ++e)
-        if (tile < full_tiles || i + e < n) flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
+        if (tile < full_tiles || i + e < n) {
+          flags |= (mag_key(a[c][e]) >= T ? 1u : 0u) << (c * 4 + e);
+          nonfinite += mag_key(a[c][e]) >= 0x7F800000u;
+        }
     }
     if (flags) {
 #pragma unroll
       for (int c = 0; c < 4; ++c)
 #pragma unroll
         for (int e = 0; e < 4; ++e)
-          if ((flags >> (c * 4 + e)) & 1u) atomicAdd(&s_h[mag_key(a[c][e]) >> shift(0)], 1u);
+          if ((flags >> (c * 4 + e)) & 1u) atomicAdd(&s_h[fine_bin(mag_key(a[c][e]), T, FS)], 1u);
     }
     uint32_t vec_base[4];
     uint64_t excl;
@@ -516,11 +560,13 @@ __global__ void __launch_bounds__(kThreads) stream_tma_kernel(const void* __rest
       uint32_t b = total ? atomicAdd(&ctl->cand_count, total) : 0u;
       s_base[par] = b;
       tile_info[tile] = make_uint2(b, total);
+      tk[tile] = 0;
     }
     __syncthreads();
     tile_tail(a, flags, total, vec_base, excl, s_base[par], cap, base, n, tile < full_tiles, vbf16, r,
               cand_idx, cand_val);
   }
+  if (nonfinite) atomicAdd(&ctl->nonfinite, nonfinite);
   __syncthreads();
   for (int j = threadIdx.x; j < bins(0); j += kThreads)
     if (s_h[j]) atomicAdd(hc + j, s_h[j]);
@@ -538,12 +584,20 @@ struct SelArgs {
   uint32_t num_tiles, cap;
   uint32_t *hs, *hc, *hc2, *h0, *h1, *h2;
   uint64_t* tloc;
+  uint64_t* tk;            // fast select: packed (> K*, == K*) counts per tile
+  uint64_t* ctot;          // fast select: the same per chunk of chunk_tiles tiles
+  uint32_t* hl;            // fast select: low key bits of the undecided
+  uint32_t* gbits;         // fast select: "> K*" bit per candidate position
+  uint32_t* ebits;         // fast select: "== K*" bit per candidate position
+  uint64_t* inbin;         // fast select: (position, value) of the undecided
+  uint32_t chunk_tiles, num_chunks;
   uint64_t* boff;
   uint8_t* pairs;
   uint32_t num_micro;       // recovery sample
   double stride, phase;
   int exhaustive;
   uint32_t force_t2;        // test hook: the rescan's threshold
+  int fast;                 // the fast select may run (LOWDIFF_FAST_SELECT=0: always the general path)
 };
 
 // One cooperative launch runs the three digit passes (12 + 10 + 9 bits of the 31-bit key) with a
@@ -752,16 +806,259 @@ __device__ void rescan(const SelArgs& A, uint32_t T2, int vbf16, float* s_ov, ui
     if (s_h[j]) atomicAdd(A.hc2 + j, s_h[j]);
 }
 
+// ---- K2 fast path: warm first pass, the k-th key in a narrow fine bin ------------------------
+// The stream pass histogrammed the candidates into fine bins relative to T (bin width 2^s keys,
+// s <= 12). The bin b* holding the k-th largest key splits the candidates: bins above b* are
+// surely > K*, bins below surely < K* (rejected), those in b* are undecided until K* is known.
+//   phase 1 (balanced over buffer positions): per position a "> K*" bit and a "== K*" bit (one
+//     warp ballot per 32 positions), packed (>, ==) counts per tile and per chunk of tiles
+//     (warp-aggregated 64-bit atomics); the undecided go to a list plus a histogram of their low
+//     s key bits; the surely rejected get r = a back.                     -- grid barrier --
+//   phase 2 (every CTA): K* and the kept tie count m from the low-bit histogram; each CTA resolves
+//     a slice of the undecided list into the bits and counts (< K*: r = a). -- grid barrier --
+//   phase 3 (balanced over positions): for the candidate at buffer position p in tile t,
+//     (gt, eq) before it = (chunk offset) + (a warp-wide sum over t's chunk before t) + (bits in t's
+//     segment before p); kept iff > K*, or == K* with eq < m; slot = gt + min(eq, m).
+// The candidates of one tile are contiguous in the buffer and in index order, so "before" is
+// "at a lower index". Two grid barriers, no tile scan (the general path has five).
+__device__ __forceinline__ uint64_t warp_sum64(uint64_t v) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, o);
+  return v;
+}
+
+template <bool VBF16>
+__device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t bst, uint64_t above,
+                            uint32_t cc, uint8_t* s_raw, uint64_t* s_scan, cg::grid_group& grid) {
+  Ctl* ctl = A.ctl;
+  const uint64_t k = A.k;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t lowmask = (1u << S) - 1;
+  const uint32_t CH = A.chunk_tiles, num_tiles = A.num_tiles;
+  constexpr uint64_t kGt = 1ull << 32;             // packed count: (> K*) << 32 | (== K*)
+  float* r = A.r;
+  const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
+  const uint64_t wid = ((uint64_t)blockIdx.x * kThreads + threadIdx.x) >> 5;
+  // ---- phase 1: classify (4 words per warp in flight) ----
+  constexpr int U1 = 4;
+  for (uint64_t base0 = wid * 32; base0 < cc; base0 += U1 * nwarps * 32) {   // warp-uniform
+  float av[U1];
+  uint32_t iv[U1];
+#pragma unroll
+  for (int v = 0; v < U1; ++v) {
+    const uint64_t pv = base0 + v * nwarps * 32 + lane;
+    av[v] = pv < cc ? A.cval1[pv] : 0.f;
+    iv[v] = pv < cc ? A.cidx1[pv] : 0u;
+  }
+#pragma unroll
+  for (int u = 0; u < U1; ++u) {
+    const uint64_t base = base0 + u * nwarps * 32;
+    if (base >= cc) break;                         // warp-uniform
+    const uint64_t p = base + lane;
+    const bool in = p < cc;
+    const float a = av[u];
+    const uint32_t idx = iv[u];
+    const uint32_t key = mag_key(a);
+    const uint32_t fb = in ? fine_bin(key, T, S) : 0u;
+    const bool sure = in && fb > bst, und = in && fb == bst;
+    if (in && fb < bst) r[idx] = a;                // surely rejected: keeps all of a
+    const uint32_t sk = __ballot_sync(0xFFFFFFFFu, sure);
+    if (lane == 0) { A.gbits[base >> 5] = sk; A.ebits[base >> 5] = 0u; }
+    if (sure) {                                    // one atomic per tile (and chunk) per warp
+      const uint32_t tile = idx / kTile;
+      const uint32_t peers = __match_any_sync(sk, tile);
+      if (lane == __ffs(peers) - 1) {
+        atomicAdd(reinterpret_cast<unsigned long long*>(&A.tk[tile]), (unsigned long long)__popc(peers) << 32);
+        atomicAdd(reinterpret_cast<unsigned long long*>(&A.ctot[tile / CH]), (unsigned long long)__popc(peers) << 32);
+      }
+    }
+    const uint32_t ub = __ballot_sync(0xFFFFFFFFu, und);
+    if (ub) {
+      uint32_t slot0 = 0;
+      if (lane == __ffs(ub) - 1) slot0 = atomicAdd(&ctl->inbin_count, (uint32_t)__popc(ub));
+      slot0 = __shfl_sync(0xFFFFFFFFu, slot0, __ffs(ub) - 1);
+      if (und) {
+        A.inbin[slot0 + __popc(ub & ((1u << lane) - 1))] = ((uint64_t)p << 32) | __float_as_uint(a);
+        atomicAdd(&A.hl[(key - T) & lowmask], 1u);
+      }
+    }
+  }
+  }
+  grid.sync();
+  // ---- phase 2: K*, m; resolve this CTA's slice of the undecided ----
+  __shared__ uint32_t s_K;
+  __shared__ uint64_t s_m;
+  const uint64_t need = k - above;                 // rank of K* inside bin b* (>= 1)
+  {
+    const uint32_t NB = 1u << S;
+    const uint32_t per = NB > kThreads ? NB / kThreads : 1;
+    const bool act = threadIdx.x * per < NB;
+    const uint32_t lo = act ? NB - (threadIdx.x + 1) * per : 0;
+    uint64_t sum = 0;
+    for (uint32_t q = 0; q < per && act; ++q) sum += __ldcg(A.hl + lo + q);
+    uint64_t tot;
+    uint64_t ab = block_exclusive_scan(sum, s_scan, &tot);
+    if (act && ab < need && ab + sum >= need) {
+      for (int q = (int)per - 1; q >= 0; --q) {
+        const uint32_t c = __ldcg(A.hl + lo + q);
+        if (ab + c >= need) { s_K = T + (bst << S) + lo + q; s_m = need - ab; break; }
+        ab += c;
+      }
+    }
+    __syncthreads();
+  }
+  const uint32_t K = s_K;
+  const uint64_t m = s_m;
+  const uint32_t n_in = __ldcg(&ctl->inbin_count);
+  for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < n_in; i += (uint64_t)gridDim.x * kThreads) {
+    const uint64_t e = __ldcg(A.inbin + i);
+    const uint32_t p = (uint32_t)(e >> 32);
+    const float a = __uint_as_float((uint32_t)e);
+    const uint32_t key = mag_key(a), idx = A.cidx1[p];
+    if (key >= K) {
+      const uint64_t inc = key > K ? kGt : 1ull;
+      atomicOr(key > K ? &A.gbits[p >> 5] : &A.ebits[p >> 5], 1u << (p & 31));
+      atomicAdd(reinterpret_cast<unsigned long long*>(&A.tk[idx / kTile]), (unsigned long long)inc);
+      atomicAdd(reinterpret_cast<unsigned long long*>(&A.ctot[idx / kTile / CH]), (unsigned long long)inc);
+    } else {
+      r[idx] = a;                                  // below K*: keeps all of a
+    }
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    ctl->mode = 3; ctl->kstar = K; ctl->m = m;
+    state_update(A.st, A.sk, k, A.cap, cc, 3, K, ctl->nonfinite);
+  }
+  grid.sync();
+  // ---- phase 3: chunk offsets (every CTA), then the ordered emission ----
+  uint64_t* s_coff = reinterpret_cast<uint64_t*>(s_raw);          // <= 4096 chunks
+  {
+    const uint32_t nch = A.num_chunks;
+    const uint32_t per = (nch + kThreads - 1) / kThreads;         // <= 16
+    uint64_t v[16], gsum = 0, esum = 0;
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      const uint32_t c = threadIdx.x * per + q;
+      v[q] = (q < (int)per && c < nch) ? __ldcg(A.ctot + c) : 0ull;
+      gsum += v[q] >> 32;
+      esum += v[q] & 0xFFFFFFFFull;
+    }
+    uint64_t tot;
+    uint64_t run = block_exclusive_scan((gsum << 32) | esum, s_scan, &tot);   // both halves < 2^32
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      const uint32_t c = threadIdx.x * per + q;
+      if (q < (int)per && c < nch) s_coff[c] = run;
+      run += v[q];
+    }
+  }
+  __syncthreads();
+  uint8_t* pairs = A.pairs;
+  uint32_t* out_idx = reinterpret_cast<uint32_t*>(pairs);
+  uint8_t* out_val = pairs + pad16(4 * k);
+  if (blockIdx.x == 0 && threadIdx.x < 16) {       // zero the 16-byte padding of both sections
+    const uint64_t ip = 4 * k, ie = pad16(4 * k);
+    if (ip + threadIdx.x < ie) pairs[ip + threadIdx.x] = 0;
+    const uint64_t vp = pad16(4 * k) + (VBF16 ? 2 : 4) * k, ve = pad16(4 * k) + pad16((VBF16 ? 2 : 4) * k);
+    if (vp + threadIdx.x < ve) pairs[vp + threadIdx.x] = 0;
+  }
+  // Warps take runs of W consecutive 32-position words (runs strided over the grid), carrying the
+  // packed (gt, eq) count of the current tile from word to word: a tile's prefix (chunk offset + a
+  // warp-wide sum over its chunk) is computed once per tile a run meets, the segment carry before
+  // the run (a warp-wide popcount over earlier words) once per run. Long runs amortise that when
+  // tiles hold many candidates, but serialise the warp.
+  const uint32_t lt = (1u << lane) - 1;
+  // (measured: one word per run when tiles hold < 32 candidates, C2/C3; one contiguous range per
+  // warp above, C4)
+  const uint64_t W = (cc / (num_tiles ? num_tiles : 1)) >= 32 ? ((cc + nwarps * 32 - 1) / (nwarps * 32)) : 1;
+  for (uint64_t run0 = wid * 32 * W; run0 < cc; run0 += nwarps * 32 * W) {   // warp-uniform
+  const uint64_t p_end = run0 + 32 * W < cc ? run0 + 32 * W : cc;
+  uint32_t cur_t = 0xFFFFFFFFu;                    // the tile continuing from the previous word
+  uint64_t cur_before = 0;                         // its packed (gt, eq) before the current word
+  auto tile_prefix = [&](uint32_t tt) -> uint64_t {   // packed count in tiles before tt (warp-wide)
+    const uint32_t cb = tt / CH * CH;
+    uint64_t part = 0;
+    for (uint32_t j = cb + lane; j < tt; j += 32) part += __ldcg(A.tk + j);
+    return warp_sum64(part) + s_coff[tt / CH];
+  };
+  // the next word's loads are issued before the current word is processed
+  uint32_t n_idx = 0, n_gw = 0, n_ew = 0;
+  float n_a = 0.f;
+  auto load_word = [&](uint64_t bw) {
+    const uint64_t pw = bw + lane;
+    n_idx = pw < p_end ? A.cidx1[pw] : 0u;
+    n_a = pw < p_end ? A.cval1[pw] : 0.f;
+    n_gw = bw < p_end ? __ldcg(A.gbits + (bw >> 5)) : 0u;
+    n_ew = bw < p_end ? __ldcg(A.ebits + (bw >> 5)) : 0u;
+  };
+  load_word(run0);
+  for (uint64_t base = run0; base < p_end; base += 32) {   // warp-uniform
+    const uint64_t p = base + lane;
+    const bool in = p < p_end;
+    const uint32_t idx = n_idx, gw = n_gw, ew = n_ew;
+    const float a = n_a;
+    if (base + 32 < p_end) load_word(base + 32);
+    const uint32_t t = in ? idx / kTile : 0xFFFFFFFFu;
+    uint32_t pend = __ballot_sync(0xFFFFFFFFu, in);
+    uint64_t before = 0;
+    uint32_t last_t = 0xFFFFFFFFu;
+    uint64_t last_before = 0;
+    while (pend) {                                 // warp-uniform: each distinct tile of this word
+      const int l0 = __ffs(pend) - 1;
+      const uint32_t tt = __shfl_sync(0xFFFFFFFFu, t, l0);
+      const uint32_t same = __ballot_sync(0xFFFFFFFFu, t == tt);
+      pend &= ~same;
+      uint64_t b0;                                 // packed count before this word's first lane of tt
+      if (tt == cur_t) {
+        b0 = cur_before;
+      } else {
+        b0 = tile_prefix(tt);
+        const uint32_t sx = A.tinfo1[tt].x;
+        if (sx < base) {                           // only at the range start: the segment began earlier
+          uint64_t c = 0;
+          for (uint64_t w = (sx >> 5) + lane; w < (base >> 5); w += 32) {
+            uint32_t g1 = __ldcg(A.gbits + w), e1 = __ldcg(A.ebits + w);
+            if (w == (sx >> 5)) { g1 &= ~((1u << (sx & 31)) - 1); e1 &= ~((1u << (sx & 31)) - 1); }
+            c += ((uint64_t)__popc(g1) << 32) | __popc(e1);
+          }
+          b0 += warp_sum64(c);
+        }
+      }
+      const uint32_t lanes_lt_first = (1u << l0) - 1;   // tt's lanes are contiguous from l0
+      if ((same >> lane) & 1u) {
+        const uint32_t msk = lt & ~lanes_lt_first;
+        before = b0 + (((uint64_t)__popc(gw & msk)) << 32) + __popc(ew & msk);
+      }
+      last_t = tt;
+      last_before = b0 + (((uint64_t)__popc(gw & same)) << 32) + __popc(ew & same);
+    }
+    cur_t = last_t;                                // the word's last tile may continue
+    cur_before = last_before;
+    const bool isg = in && ((gw >> lane) & 1u), ise = in && ((ew >> lane) & 1u);
+    const uint64_t gtb = before >> 32, eqb = before & 0xFFFFFFFFull;
+    if (isg || (ise && eqb < m)) {
+      const uint64_t pos = gtb + (eqb < m ? eqb : m);
+      out_idx[pos] = idx;
+      if constexpr (VBF16) reinterpret_cast<__nv_bfloat16*>(out_val)[pos] = __float2bfloat16_rn(a);
+      else reinterpret_cast<float*>(out_val)[pos] = a;
+    } else if (ise) {
+      r[idx] = a;                                  // a tie beyond the m kept: keeps all of a
+    }
+  }
+  }
+}
+
 template <bool VBF16>
 __global__ void __launch_bounds__(kThreads, 4) select_kernel(SelArgs A) {
   cg::grid_group grid = cg::this_grid();
-  __shared__ uint32_t sh[bins(0)];
+  __shared__ __align__(16) uint8_t s_raw[2 * 4 * kTile];    // general: histogram | recovery overlay
   __shared__ uint64_t s_scan[2][kThreads / 32];
+  uint32_t* sh = reinterpret_cast<uint32_t*>(s_raw);
   Ctl* ctl = A.ctl;
   if (ctl->small_done) return;                     // the one-CTA select did this call (uniform)
   const uint64_t n = A.n, k = A.k;
   const uint32_t cap = A.cap, num_tiles = A.num_tiles;
   const uint32_t cc = ctl->cand_count;
+  const uint32_t T = ctl->t_est, FS = ctl->fine_shift;
   // the candidate set the select runs on: the first pass's, unless it missed
   const uint32_t* cidx = A.cidx1;
   const float* cval = A.cval1;
@@ -769,20 +1066,28 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(SelArgs A) {
   const uint32_t* hfirst = A.hc;
   uint64_t N = cc;
   uint32_t mode = 0;
+  if (cc >= k && cc <= cap) {
+    uint64_t above;
+    const int bst = find_bin_desc<bins(0)>(A.hc, k, &above, s_scan[0]);
+    const uint32_t inb = bst >= 0 ? __ldcg(A.hc + bst) : ~0u;
+    if (A.fast && bst >= 0 && bst < 4095 && FS <= 12 && inb <= cap) {
+      fast_select<VBF16>(A, T, FS, (uint32_t)bst, above, cc, s_raw, s_scan[0], grid);
+      return;
+    }
+  }
   if (cc < k || cc > cap) {                        // recovery (uniform)
-    __shared__ float s_ov[kTile];
+    float* s_ov = reinterpret_cast<float*>(s_raw + 4 * kTile);
     __shared__ uint32_t s_bits[kTile / 32];
     __shared__ uint32_t s_base[2];
     __shared__ uint32_t s_t2;
-    const uint32_t T = ctl->t_est;
     bool try_rescan = true;
     if (cc > cap) {
-      // too many: the k-th key's bin in the exact first-digit histogram of ALL candidates
+      // too many: the k-th key's bin in the exact fine histogram of ALL candidates
       uint64_t above;
       const int bk = find_bin_desc<bins(0)>(A.hc, k, &above, s_scan[0]);
-      const uint32_t lo_edge = bk < 0 ? 0u : (uint32_t)bk << shift(0);
+      const uint64_t lo_edge = bk < 0 ? 0ull : (uint64_t)T + ((uint64_t)bk << FS);
       const uint64_t cnt = bk < 0 ? ~0ull : above + __ldcg(A.hc + bk);
-      if (threadIdx.x == 0) s_t2 = lo_edge > T ? lo_edge : T;
+      if (threadIdx.x == 0) s_t2 = (uint32_t)(lo_edge < 0x7FFFFFFFull ? lo_edge : 0x7FFFFFFFull);
       try_rescan = cnt <= cap;
     } else {
       // too few: a stratified sample of the keys (the first pass's candidates read as their
@@ -823,9 +1128,9 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(SelArgs A) {
   const float* src = mode == 1 ? A.r : cval;
   uint32_t prefix = 0;
   uint64_t need = k;
-  // candidate modes: the pass that built the set already histogrammed its first digit
-  select_pass<0>(src, N, sh, mode == 1 ? A.h0 : const_cast<uint32_t*>(hfirst), prefix, need, s_scan[0], grid,
-                 mode == 1);
+  // the rescan built its set's first-digit histogram; the first pass's is relative to T (fine)
+  select_pass<0>(src, N, sh, mode == 2 ? const_cast<uint32_t*>(hfirst) : A.h0, prefix, need, s_scan[0], grid,
+                 mode != 2);
   select_pass<1>(src, N, sh, A.h1, prefix, need, s_scan[0], grid);
   select_pass<2>(src, N, sh, A.h2, prefix, need, s_scan[0], grid);
   const uint32_t K = prefix;
@@ -834,10 +1139,7 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(SelArgs A) {
     ctl->mode = mode;
     ctl->kstar = K;
     ctl->m = m;
-    const uint32_t* hf = mode == 1 ? A.h0 : hfirst;
-    uint64_t nonfinite = 0;                        // keys >= +Inf: all of them are candidates
-    for (uint32_t b = kNonFiniteBin; b < (uint32_t)bins(0); ++b) nonfinite += __ldcg(hf + b);
-    state_update(A.st, A.sk, k, cap, cc, mode, K, nonfinite);
+    state_update(A.st, A.sk, k, cap, cc, mode, K, ctl->nonfinite);
   }
   // ---- fused ordered emission ----
   // A streaming tile's candidates sit contiguously in the buffer, in index order (candidate modes),
@@ -1049,13 +1351,11 @@ select_small_kernel(float* __restrict__ r, uint64_t k, Ctl* ctl, const float* __
   __shared__ uint32_t s_h0[bins(0)], s_h1[bins(1)], s_h2[bins(2)];
   __shared__ uint64_t s_scan[33];
   const uint32_t tid = threadIdx.x, lane = tid & 31;
-  for (int b = tid; b < bins(0); b += kSmallThreads) s_h0[b] = __ldcg(hc + b);
+  for (int b = tid; b < bins(0); b += kSmallThreads) s_h0[b] = 0;
   for (int b = tid; b < bins(1); b += kSmallThreads) s_h1[b] = 0;
   for (int b = tid; b < bins(2); b += kSmallThreads) s_h2[b] = 0;
   __syncthreads();
   uint64_t need = k, above;
-  const uint32_t d0 = (uint32_t)small_find<bins(0)>(s_h0, need, &above, s_scan);
-  need -= above;
   auto digit = [&](uint32_t* sh, int NBITS, uint32_t pfx, int pshift, int dshift) {
     for (uint32_t jw = tid & ~31u; jw < cc; jw += kSmallThreads) {   // warp-uniform trip count
       const uint32_t j = jw + lane;
@@ -1070,6 +1370,9 @@ select_small_kernel(float* __restrict__ r, uint64_t k, Ctl* ctl, const float* __
     }
     __syncthreads();
   };
+  digit(s_h0, 12, 0u, 31, shift(0));               // (the stream pass's histogram is relative to T)
+  const uint32_t d0 = (uint32_t)small_find<bins(0)>(s_h0, need, &above, s_scan);
+  need -= above;
   digit(s_h1, 10, d0, shift(0), shift(1));
   const uint32_t d1 = (uint32_t)small_find<bins(1)>(s_h1, need, &above, s_scan);
   need -= above;
@@ -1081,9 +1384,7 @@ select_small_kernel(float* __restrict__ r, uint64_t k, Ctl* ctl, const float* __
   const uint64_t m = need;                         // K*-ties to keep (lowest indices first)
   if (tid == 0) {
     ctl->mode = 0; ctl->kstar = K; ctl->m = m; ctl->small_done = 1;
-    uint64_t nonfinite = 0;
-    for (uint32_t b = kNonFiniteBin; b < (uint32_t)bins(0); ++b) nonfinite += s_h0[b];
-    state_update(st, sk, k, cap, cc, 0, K, nonfinite);
+    state_update(st, sk, k, cap, cc, 0, K, ctl->nonfinite);
   }
   auto flag = [&](uint32_t j) -> uint64_t {        // packed (key > K*, key == K*) of position j
     const uint32_t key = mag_key(cand_val[j]);
@@ -1246,7 +1547,7 @@ void compress_force_threshold(int which, int enable, uint32_t key) {
   (which == 0 ? g_force_t : g_force_t2) = enable ? key : kNoForce;
 }
 
-lowdiff_status compress_stats(const void* ws, uint64_t n, uint64_t k, uint64_t out[6], cudaStream_t s) {
+lowdiff_status compress_stats(const void* ws, uint64_t n, uint64_t k, uint64_t out[8], cudaStream_t s) {
   const Layout L = layout(n, k);
   Ctl c;
   LD_CUDA(cudaMemcpyAsync(&c, static_cast<const uint8_t*>(ws) + L.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s),
@@ -1254,20 +1555,23 @@ lowdiff_status compress_stats(const void* ws, uint64_t n, uint64_t k, uint64_t o
   LD_CUDA(cudaStreamSynchronize(s), "stats sync");
   out[0] = c.t_est; out[1] = c.cand_count; out[2] = c.mode; out[3] = c.kstar; out[4] = c.m;
   out[5] = L.cap;
+  out[6] = c.fine_shift;
+  out[7] = c.inbin_count;
   return LOWDIFF_OK;
 }
 
-lowdiff_status compress_counters(const void* ws, cudaStream_t s, uint64_t out[8]) {
+lowdiff_status compress_counters(const void* ws, cudaStream_t s, uint64_t out[9]) {
   State st;
   LD_CUDA(cudaMemcpyAsync(&st, ws, sizeof(State), cudaMemcpyDeviceToHost, s), "counters copy");
   LD_CUDA(cudaStreamSynchronize(s), "counters sync");
   if (st.magic != kStateMagic) {
-    for (int i = 0; i < 8; ++i) out[i] = 0;
+    for (int i = 0; i < 9; ++i) out[i] = 0;
     return LOWDIFF_OK;
   }
   out[0] = st.calls; out[1] = st.rescans; out[2] = st.fallbacks; out[3] = st.nonfinite_calls;
   out[4] = st.last_nonfinite; out[5] = st.last_cand; out[6] = st.kstar;
   out[7] = (uint64_t)((double)st.delta * 4294967296.0);     // delta in 2^-32 units
+  out[8] = st.fast_calls;
   return LOWDIFF_OK;
 }
 
@@ -1301,25 +1605,26 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   const bool bf = gdt == LOWDIFF_BF16;
   const int vbf = vdt == LOWDIFF_BF16 ? 1 : 0;
   uint32_t* hcand = reinterpret_cast<uint32_t*>(w + L.hc);
+  uint64_t* tk = reinterpret_cast<uint64_t*>(w + L.tk);
   if (use_tma) {
     int grid = stream_tma_blocks(bf);
     if ((uint32_t)grid > L.num_tiles) grid = (int)L.num_tiles;
     const int smem = stream_tma_smem(bf);
     if (bf)
       LD_LAUNCH("compress_stream", s, stream_tma_kernel<true>, grid, kThreads, smem, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, st, sk, g_force_t);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, tk, st, sk, g_force_t);
     else
       LD_LAUNCH("compress_stream", s, stream_tma_kernel<false>, grid, kThreads, smem, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, st, sk, g_force_t);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, tk, st, sk, g_force_t);
   } else {
     int grid = stream_blocks(bf);
     if ((uint32_t)grid > L.num_tiles) grid = (int)L.num_tiles;
     if (bf)
       LD_LAUNCH("compress_stream", s, stream_kernel<true>, grid, kThreads, 0, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, st, sk, g_force_t);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, tk, st, sk, g_force_t);
     else
       LD_LAUNCH("compress_stream", s, stream_kernel<false>, grid, kThreads, 0, grad, residual, n,
-                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, st, sk, g_force_t);
+                L.num_tiles, ctl, tiles, cidx, cval, L.cap, vbf, hcand, tk, st, sk, g_force_t);
   }
 
   const int sel_max = select_max_per_sm();
@@ -1349,10 +1654,27 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   A.h1 = reinterpret_cast<uint32_t*>(w + L.h1);
   A.h2 = reinterpret_cast<uint32_t*>(w + L.h2);
   A.tloc = reinterpret_cast<uint64_t*>(w + L.tloc);
+  A.tk = tk;
+  A.ctot = reinterpret_cast<uint64_t*>(w + L.ctot);
+  A.hl = reinterpret_cast<uint32_t*>(w + L.hl);
+  A.gbits = reinterpret_cast<uint32_t*>(w + L.bits);
+  A.ebits = A.gbits + (L.cap / 32 + 1);
+  A.inbin = reinterpret_cast<uint64_t*>(w + L.inbin);
+  {
+    const uint32_t q = (L.num_tiles + 32u * kMaxChunks - 1) / (32u * kMaxChunks);
+    A.chunk_tiles = 32u * (q ? q : 1u);
+    A.num_chunks = (L.num_tiles + A.chunk_tiles - 1) / A.chunk_tiles;
+  }
   A.boff = reinterpret_cast<uint64_t*>(w + L.boff);
   A.pairs = static_cast<uint8_t*>(pairs);
   A.num_micro = micro; A.stride = stride; A.phase = phase; A.exhaustive = exhaustive;
   A.force_t2 = g_force_t2;
+  static int use_fast = -1;
+  if (use_fast < 0) {
+    const char* e = getenv("LOWDIFF_FAST_SELECT");
+    use_fast = e ? atoi(e) : 1;
+  }
+  A.fast = use_fast;
   ProfScope prof("compress_select", s);
   static int use_small = -1;
   if (use_small < 0) {

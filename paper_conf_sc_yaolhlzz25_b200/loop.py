@@ -7,9 +7,10 @@ Per iteration t (one call of `LowDiffLoop.step(grad)`), all on the training stre
   2. live update M_{t+1} = M_t + Opt(G~_t) on this rank's shard: lowdiff_update — the replay
      kernel on G~_t as a one-iteration differential, so recovery reproduces the live trajectory
      bit for bit (Finding 1)
-  3. the Reusing Queue: G~_t stays in its own ring slot (no copy of its values); every
-     B iterations the batch is merged into one record on the training stream (§4.2)
-     into one of two device record buffers
+  3. the Reusing Queue: G~_t stays in its own ring slot (no copy of its values); when
+     lowdiff_plan_record_due says so — every B iterations, and right before every full checkpoint
+     (a short record, reading #25) — the batch is merged into one record on the training
+     stream (§4.2) into one of two device record buffers
   4. the checkpoint side (`_service`, run by the host at the start of each step): once a merge has
      finished (event query, never a wait) the record's byte count is read from pinned memory and
      the record is staged D2H on a copy stream into a pinned buffer from a reused pool (the
@@ -18,6 +19,14 @@ Per iteration t (one call of `LowDiffLoop.step(grad)`), all on the training stre
      the shard state (D2D on the training stream), then D2H on the copy stream (CheckFreq-style
      snapshot -> persist). Older full checkpoints and the records before them are
      released once a newer full checkpoint is on the host (`retain_fulls`; None keeps all).
+     Any full_every works: the record-boundary policy is the C ABI's lowdiff_plan_record_due.
+
+World > 1 (ZeRO-style reading of §8(e)): rank p owns the optimizer state of the shard [lo, hi) of
+the flat parameter vector and updates it from the coalesced G~_t of that shard. The shard state
+lives in its own (256-byte aligned) buffers; after each update it is copied into x[lo:hi] and, if
+a torch.distributed process group is given (`param_group`), the updated shards are all-gathered
+into every rank's x (parameter re-replication, plumbing outside the checkpoint path). Without a
+group only x[lo:hi] is current on this rank.
 
 `recover(t)` rebuilds the state at iteration t from the latest full checkpoint at or before t
 and the staged records after it (Alg. 1 lines 16-24): host -> device loads, then lowdiff_replay.
@@ -30,8 +39,8 @@ from __future__ import annotations
 import numpy as np
 import torch
 
-from . import (LowDiffError, allgather_sparse, batch_merge, compress, k_for_density, pairs_bytes, pairs_views,
-               record_max_bytes, replay, shard_bounds, stage_d2h, update)
+from . import (LowDiffError, allgather_sparse, batch_merge, compress, pairs_bytes, pairs_views, plan_init,
+               plan_record_due, record_max_bytes, replay, stage_d2h, update)
 
 _STATE_KEYS = ("x", "m", "v")
 
@@ -39,21 +48,23 @@ _STATE_KEYS = ("x", "m", "v")
 class LowDiffLoop:
     def __init__(self, x: torch.Tensor, opt: dict, lr: float, rho: float, B: int, full_every: int,
                  comm=None, rank: int = 0, world: int = 1, adam_step: int = 0, checkpoint: bool = True,
-                 retain_fulls: int | None = 2):
+                 retain_fulls: int | None = 2, param_group=None):
         assert x.dtype == torch.float32 and x.is_cuda and x.dim() == 1
-        assert full_every % B == 0, "full checkpoints fall on batch boundaries (records chain from them)"
         assert retain_fulls is None or retain_fulls >= 1
         self.n = x.numel()
-        self.k = k_for_density(self.n, rho)
-        self.lo, self.hi = shard_bounds(self.n, world, rank)
+        self.plan = plan_init(self.n, rho, B, full_every, "f32", "f32", world, rank)
+        self.k, self.lo, self.hi = self.plan.k, self.plan.lo, self.plan.hi
         self.world, self.comm, self.opt = world, comm, dict(opt)
+        self.x_full, self.param_group = x, param_group
         self.lr = float(np.float32(lr))
         self.B, self.full_every, self.retain_fulls = B, full_every, retain_fulls
         dev = x.device
         self.r = torch.zeros(self.n, device=dev)                      # EF residual
         L = self.hi - self.lo
         kind = opt["kind"]
-        self.state = {"x": x[self.lo:self.hi], "m": None if kind == "sgd" else torch.zeros(L, device=dev),
+        # world 1: the state IS x; world > 1: the shard in its own aligned buffer (lo % 4 may be != 0)
+        xs = x if world == 1 else x[self.lo:self.hi].clone()
+        self.state = {"x": xs, "m": None if kind == "sgd" else torch.zeros(L, device=dev),
                       "v": torch.zeros(L, device=dev) if kind == "adam" else None, "x_bf16": None,
                       "n": self.n, "lo": self.lo, "hi": self.hi, "t": 0, "adam_step": adam_step,
                       "momentum_initialized": 0}
@@ -100,29 +111,51 @@ class LowDiffLoop:
             self.full_pool = [{k: torch.empty(L, dtype=torch.float32, pin_memory=True) for k in keys}
                               for _ in range(retain_fulls + 1)]
             self.pool = [torch.empty(self.rec_cap, dtype=torch.uint8, pin_memory=True)
-                         for _ in range(min(retain_fulls * (full_every // B) + 2, 16))]   # more on demand
+                         for _ in range(min(retain_fulls * (-(-max(full_every, 1) // B)) + 2, 16))]   # more on demand
 
     # ---- one training iteration ---------------------------------------------------------------
     def step(self, grad: torch.Tensor):
+        close, _, full_due = plan_record_due(self.plan, self.t)
         if self.checkpoint:
             self._service()
-            if self.t % self.full_every == 0:
+            if full_due:
                 self._full_checkpoint()
-        idx, val, nnz = self.slots[self.t % len(self.slots)]
+        slot = len(self.ring) % len(self.slots)                         # the open record's next slot
+        idx, val, nnz = self.slots[slot]
         if self.zero_copy:
-            compress(grad, self.r, self.k, pairs=self.pair_slots[self.t % len(self.slots)])
+            compress(grad, self.r, self.k, pairs=self.pair_slots[slot])
         else:
             pairs = compress(grad, self.r, self.k, pairs=self.pairs)
             allgather_sparse(self.comm, pairs, self.k, "f32", self.lo, self.hi, out_idx=idx, out_val=val,
                              d_nnz=nnz)
         g_t = (idx, val, nnz, self.cap, self.lr)
         update(self.state, self.opt, g_t)                               # live M_{t+1}
+        if self.world > 1:
+            self._replicate()
         self.t += 1
         if not self.checkpoint:
             return
         self.ring.append(g_t)                                           # Q.put: zero copy
-        if len(self.ring) == self.B:
+        if close:                                                       # every B, and before a full checkpoint
             self._close_batch()
+
+    def _replicate(self):
+        """x[lo:hi] <- the updated shard; with a process group, all-gather every rank's shard."""
+        self.x_full[self.lo:self.hi].copy_(self.state["x"])
+        if self.param_group is None:
+            return
+        import torch.distributed as dist
+        P = self.world
+        S = -(-self.n // P) + 1                                         # shards differ by at most 1
+        if not hasattr(self, "_gbuf"):
+            self._gbuf = torch.empty(P * S, device=self.x_full.device)
+            self._mine = torch.empty(S, device=self.x_full.device)
+        self._mine[:self.hi - self.lo].copy_(self.state["x"])
+        dist.all_gather_into_tensor(self._gbuf, self._mine, group=self.param_group)
+        for p in range(P):
+            lo, hi = p * self.n // P, (p + 1) * self.n // P
+            if p != self.plan.rank:
+                self.x_full[lo:hi].copy_(self._gbuf[p * S:p * S + hi - lo])
 
     def _close_batch(self):
         d = self.drec[self.next_drec]
@@ -218,7 +251,7 @@ class LowDiffLoop:
 
     # ---- recovery (Alg. 1 lines 16-24) -----------------------------------------------------------
     def recover(self, t: int) -> dict:
-        """State of this shard at iteration t (t a batch boundary), from the latest full checkpoint
+        """State of this shard at iteration t (t a record boundary), from the latest full checkpoint
         at or before t and the staged records after it, loaded back from the host."""
         self.flush()
         tf, snap, _ = max((f for f in self.fulls if f[0] <= t), key=lambda f: f[0])

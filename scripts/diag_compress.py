@@ -37,6 +37,7 @@ for it in range(a.iters):
         f = lambda key: struct.unpack("<f", struct.pack("<I", int(key)))[0]
         print(f"it {it:4d} cand/k {st['candidates'] / cfg.k:7.3f} cap/k {st['capacity'] / cfg.k:6.2f} "
               f"path {st['path']} t_est {f(st['t_est']):.6g} kstar {f(st['kstar']):.6g} "
-              f"ratio {f(st['t_est']) / max(f(st['kstar']), 1e-30):.4f}", flush=True)
+              f"ratio {f(st['t_est']) / max(f(st['kstar']), 1e-30):.4f} S {st['fine_shift']} inbin {st['inbin']} "
+              f"ties {st['ties_kept']}", flush=True)
 print(f"fallbacks: {fallbacks} rescans: {rescans} / {a.iters}")
 print(ld.compress_counters(cfg.n, cfg.k))
