@@ -61,19 +61,21 @@ def parse_args():
 # ---------------------------------------------------------------------------------------------
 # CPU oracle arm (cpu_baseline and --impl reference): the oracle as it stands, bounded sample
 # ---------------------------------------------------------------------------------------------
-def oracle_step_sample(cfg, n_s: int, t0: int = 0):
+def oracle_step_sample(cfg, n_s: int, t0: int = 0, grads=None):
     """Time the oracle on one step of the same workload restricted to the first n_s gradient
     elements (same rho, B, chain length, optimizer): R = K/B batches of B compress + coalesce and
-    one merge each, then one replay of the R-record chain. Returns (seconds, gradient bytes)."""
+    one merge each, then one replay of the R-record chain. `grads`: host copies of the GPU arm's own
+    gradient tensors (same values); else drawn on the CPU. Returns (seconds, gradient bytes)."""
     import numpy as np
     import oracle
     from workloads import gradient, segment_sigmas
     import torch
-    sig = segment_sigmas(cfg)[:n_s]
     k = max(1, int(cfg.rho * n_s))
     R = chain_records(cfg)
-    grads = [gradient(cfg, 0, t0 + t, "cpu", sigmas=sig, n=n_s) for t in range(cfg.B)]
-    grads = [g.view(torch.int16).numpy().view(np.uint16) if cfg.gdt == "bf16" else g.numpy() for g in grads]
+    if grads is None:
+        sig = segment_sigmas(cfg)[:n_s]
+        grads = [gradient(cfg, 0, t0 + t, "cpu", sigmas=sig, n=n_s) for t in range(cfg.B)]
+        grads = [g.view(torch.int16).numpy().view(np.uint16) if cfg.gdt == "bf16" else g.numpy() for g in grads]
     r = np.zeros(n_s, np.float32)
     lr = np.float32(cfg.hyper["lr"])
     x = np.zeros(n_s, np.float32); m = np.zeros(n_s, np.float32); v = np.zeros(n_s, np.float32)
@@ -96,6 +98,43 @@ def oracle_step_sample(cfg, n_s: int, t0: int = 0):
     return dt, gbytes
 
 
+def host_description() -> dict:
+    """nproc and the CPU model of the host the oracle runs on."""
+    model = None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    try:
+        avail = len(os.sched_getaffinity(0))
+    except AttributeError:
+        avail = os.cpu_count()
+    return {"nproc": avail, "cpu_model": model}
+
+
+def _oracle_worker(args):
+    cfg_id, n_s, grads = args
+    from workloads import CONFIGS
+    dt, gb = oracle_step_sample(CONFIGS[cfg_id], n_s, grads=grads)
+    return dt, gb
+
+
+def oracle_all_cores(cfg, n_s: int, grads, procs: int) -> dict:
+    """The same bounded step as `procs` independent oracle processes at once (independent units, as
+    P data-parallel ranks would be): aggregate gradient GB/s over the wall time."""
+    import multiprocessing as mp
+    ctx = mp.get_context("fork")
+    t0 = time.perf_counter()
+    with ctx.Pool(procs) as pool:
+        res = pool.map(_oracle_worker, [(cfg.cid, n_s, grads)] * procs)
+    wall = time.perf_counter() - t0
+    return {"value": sum(gb for _, gb in res) / wall / 1e9, "unit": "GB/s", "processes": procs,
+            "wall_s": wall}
+
+
 def chain_records(cfg) -> int:
     """Records per step: the config's replay chain of K differentials is K/B batch records."""
     return max(1, cfg.K // cfg.B)
@@ -105,25 +144,35 @@ def run_reference(args, cfg):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return  # rank 0 alone runs the CPU oracle arm
-    n_s = max(1 << 16, cfg.n // 64)
+    import numpy as np
+    import torch
+    from workloads import gradient, segment_sigmas
+    n_s = max(1 << 16, cfg.n // 16)                    # the same bounded sample as the GPU arm's cpu_baseline
+    # the GPU arm's own gradient values: drawn with the CUDA generator when a GPU is present
+    dev = "cuda" if torch.cuda.is_available() else "cpu"
+    sig = segment_sigmas(cfg, dev)[:n_s]
+    grads = [gradient(cfg, 0, t, dev, sigmas=sig, n=n_s) for t in range(cfg.B)]
+    grads = [g.view(torch.int16).cpu().numpy().view(np.uint16) if cfg.gdt == "bf16" else g.cpu().numpy()
+             for g in grads]
     for w in range(args.warmup):
-        oracle_step_sample(cfg, n_s, t0=0)
+        oracle_step_sample(cfg, n_s, grads=grads)
     times, gb = [], 0
     for s in range(args.steps):
-        dt, gb = oracle_step_sample(cfg, n_s, t0=0)
+        dt, gb = oracle_step_sample(cfg, n_s, grads=grads)
         times.append(dt)
     tot = sum(times)
     val = args.steps * gb / tot / 1e9
     sample = (f"oracle (plain C++, 1 thread) full step of {cfg.name} on the first {n_s} of n={cfg.n} "
               f"gradient elements (rho={cfg.rho}, {chain_records(cfg)} batches of B={cfg.B}, {cfg.opt} replay "
-              f"of the {cfg.K}-iteration chain)")
+              f"of the {cfg.K}-iteration chain; gradients from the {dev.upper()} generator, the GPU arm's values)")
     line = {"impl": "reference", "metric": "diff-build & replay gradient GB/s at 1/2/4/8 B200, % of HBM roofline",
             "value": val, "unit": "GB/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1e3 * tot / args.steps, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f32" if cfg.gdt == "f32" else "bf16", "data": "synthetic",
             "config": {"workload": cfg.name, "n": cfg.n, "n_sample": n_s, "rho": cfg.rho, "B": cfg.B,
                        "replay": f"{cfg.opt}, chain of {cfg.K} iterations ({chain_records(cfg)} records)"},
-            "cpu_baseline": {"value": val, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": val, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample,
+                             **host_description()},
             "e2e": {"value": val, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -219,9 +268,11 @@ def run_ours(args, cfg):
     # recovery, Load(C^F_t) + replay of the batch's record (Alg.1 l.16-24), read from the checkpoint
     # and written to the state buffers (out of place: same HBM traffic as in place).
     ck = full_checkpoint(cfg, lo, hi, dev)
+    # C4 (bf16 gradients, fp32 master): the replay also writes the bf16 copy of x
+    xb = torch.empty(hi - lo, dtype=torch.bfloat16, device=dev) if cfg.gdt == "bf16" else None
     state = {"x0": ck["x"], "m0": ck["m"], "v0": ck["v"],
              "x": torch.empty_like(ck["x"]), "m": None if ck["m"] is None else torch.empty_like(ck["m"]),
-             "v": None if ck["v"] is None else torch.empty_like(ck["v"]), "x_bf16": None, "n": n, "lo": lo,
+             "v": None if ck["v"] is None else torch.empty_like(ck["v"]), "x_bf16": xb, "n": n, "lo": lo,
              "hi": hi, "t": 0, "adam_step": ck["adam_step"], "momentum_initialized": ck["momentum_initialized"]}
     opt = {"kind": cfg.opt, **{kk: vv for kk, vv in cfg.hyper.items() if kk != "lr"}}
     lr = float(np.float32(cfg.hyper["lr"]))
@@ -423,6 +474,7 @@ def run_ours(args, cfg):
     if rp_n:
         nloc = hi - lo
         sb = {"sgd": 8, "momentum": 16, "adam": 24}[cfg.opt]          # read + write of x (m, v)
+        sb += 2 if xb is not None else 0                                 # + the bf16 copy of x (C4)
         alg = sb * nloc + int(rec_bytes)                                 # + the chain's records
         t_s = rp_ms / args.steps * 1e-3                                  # per step (one chain)
         replay_roof = {"kernel": "replay_dense", "alg_bytes_per_step": alg,
@@ -492,6 +544,7 @@ def run_ours(args, cfg):
 
     # ---- e2e: same metric through the public API with host buffers (pinned H2D of every gradient) ----
     e2e = None
+    cpu_grads = grads[:2]                               # kept for the CPU baseline (same values)
     if not args.no_e2e:
         npool = min(B, 2)
         hpool = [torch.empty(n, dtype=grads[0].dtype, pin_memory=True) for _ in range(npool)]
@@ -510,14 +563,45 @@ def run_ours(args, cfg):
                "h2d_bytes_per_step": R * B * n * gsz, "d2h_bytes_per_step": int(enb) + R * (80 + 4 * B + 8),
                "ms_per_step": e_ms, "steps": e_steps}
 
-    # ---- CPU oracle baseline (rank 0, N = 1 only) ----
+    # ---- CPU oracle baseline (rank 0, N = 1 only), on the GPU arm's own gradient values ----
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
         n_s = max(1 << 16, cfg.n // 16)
-        dt, gb = oracle_step_sample(cfg, n_s)
+        hgr = [(gg[:n_s].view(torch.int16).cpu().numpy().view(np.uint16) if cfg.gdt == "bf16"
+                else gg[:n_s].cpu().numpy()) for gg in cpu_grads]
+        hgr = [hgr[t % len(hgr)] for t in range(B)]
+        dts = []
+        for _ in range(2):
+            dt, gb = oracle_step_sample(cfg, n_s, grads=hgr)
+            dts.append(dt)
+        dt = min(dts)
+        host = host_description()
         cpu = {"value": gb / dt / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
-               "sample": f"one full step of {cfg.name} on the first {n_s} of n={cfg.n} elements "
-                         f"(B={cfg.B} compress+coalesce, merge, {cfg.opt} replay), {dt:.1f} s"}
+               "sample": f"one full step of {cfg.name} on the first {n_s} of n={cfg.n} elements of the GPU "
+                         f"arm's own gradient tensors (B={cfg.B} compress+coalesce, merge, {cfg.opt} replay), "
+                         f"best of 2: {dt:.1f} s",
+               **host}
+        try:
+            cpu["all_cores"] = oracle_all_cores(cfg, n_s, hgr, max(1, min(host["nproc"] or 1, 16)))
+        except Exception as e:                          # pragma: no cover
+            cpu["all_cores"] = {"error": str(e)[:200]}
+        # one full-n compress step on the GPU's exact inputs (its gradient and current residual):
+        # the oracle's time for that step, and the GPU's output for the same inputs compared bytewise
+        g_full, r_dev = cpu_grads[0], r.clone()
+        g_np = g_full.view(torch.int16).cpu().numpy().view(np.uint16) if cfg.gdt == "bf16" else g_full.cpu().numpy()
+        r_np = r_dev.cpu().numpy()
+        ovd = oracle.BF16 if cfg.vdt == "bf16" else oracle.F32
+        t0 = time.perf_counter()
+        oi, ov, ro = oracle.compress(g_np, r_np, k, ovd)
+        t_c = time.perf_counter() - t0
+        pairs_chk = ld.compress(g_full, r_dev, k, vdt=cfg.vdt)
+        same = bool(np.array_equal(pairs_chk.cpu().numpy(), oracle.pairs_pack(oi, ov, ovd)) and
+                    np.array_equal(r_dev.cpu().numpy().view(np.uint32), ro.view(np.uint32)))
+        cpu["compress_full_n"] = {"value": n * gsz / t_c / 1e9, "unit": "GB/s", "seconds": t_c,
+                                  "gpu_equals_oracle": same,
+                                  "sample": "one compress of the full gradient at the bench's EF state "
+                                            "(D2H copies of the GPU's g and residual)"}
 
     if p2p is not None:                                 # a timed-out peer wait voids the numbers
         torch.cuda.synchronize()
