@@ -359,7 +359,7 @@ def run_ours(args, cfg):
         state["t"] = t_iter[0] - R * B                  # the checkpoint is stamped at the chain start
         state["adam_step"] = ck["adam_step"]
         state["momentum_initialized"] = ck["momentum_initialized"]
-        ld.replay(state, opt, [(records[b], heads[b]) for b in range(R)])
+        ld.replay(state, opt, [(records[b], heads[b]) for b in range(R)], check=False)
         main.wait_stream(copy_stream)
 
     def step(graph=None, h2d=None):
@@ -423,6 +423,7 @@ def run_ours(args, cfg):
     launches0 = ld.launch_count()
     cc0 = ld.compress_counters(ws=cws)
     ms, rec_bytes = timed(args.steps, graph=graph)
+    ld.replay_check()                                   # no record body failed device validation
     cc1 = ld.compress_counters(ws=cws)
     launches = ld.launch_count() - launches0 + (graph_launches * args.steps if graph is not None else 0)
     clk = clocks.stop()

@@ -297,7 +297,8 @@ lowdiff_status lowdiff_stage_d2h(const void* d_record, uint64_t bytes, void* h_p
  *     x0/m0/v0: optional full checkpoint C^F_t to load from (Alg.1 line 17, M_t <- Load(C^F_t)):
  *     when set, the replay reads the starting state from them and writes the result to x/m/v
  *     (same HBM traffic as in place; the checkpoint stays untouched). NULL = in place.
- * Errors: ECHAIN (t gap/overlap, n/lo/hi/nranks mismatch), ECORRUPT (header), EUNSUPPORTED.
+ * Errors: ECHAIN (t gap/overlap, n/lo/hi/nranks mismatch), ECORRUPT (header; the body through
+ *   lowdiff_replay_check), EUNSUPPORTED.
  * ------------------------------------------------------------------------------------------- */
 typedef struct {
   int32_t kind;                       /* lowdiff_opt_kind */
@@ -327,6 +328,15 @@ lowdiff_status lowdiff_replay_workspace_size(const lowdiff_state* st, const lowd
 lowdiff_status lowdiff_replay(lowdiff_state* st, const lowdiff_opt* opt,
                               const lowdiff_record_view* recs, uint32_t nrec, void* ws,
                               uint64_t ws_bytes, lowdiff_stream_t stream);
+/* Device validation of the record bodies (a record damaged in storage is what recovery reads):
+ * before any replay kernel reads a body, one pass checks that the device header equals the host
+ * copy the call was planned from, lo <= idx < hi strictly ascending, and for STACK off[0] = 0,
+ * off strictly increasing to off[nnz] = nent, it[] < B strictly increasing within each index.
+ * On failure every replay kernel of the call returns without writing (the state is unchanged, no
+ * index is used out of bounds). lowdiff_replay_check(ws) synchronizes `stream` and returns
+ * ECORRUPT if the last lowdiff_replay with this workspace failed validation (lowdiff_replay itself
+ * does not synchronize). lowdiff_replay_parallel validates and checks synchronously itself. */
+lowdiff_status lowdiff_replay_check(const void* ws, lowdiff_stream_t stream);
 
 /* ---------------------------------------------------------------------------------------------
  * (5c) Live update — Alg.1 training process, "G_t <- Comp^{-1}(G~_t)" and "M_{t+1} <- M_t +

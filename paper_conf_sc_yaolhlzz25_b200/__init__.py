@@ -90,7 +90,7 @@ EXPORTS = [
     "lowdiff_update_workspace_size", "lowdiff_update", "lowdiff_dense_update", "lowdiff_host_update",
     "lowdiff_p2p_window_bytes", "lowdiff_p2p_export_handle", "lowdiff_p2p_init", "lowdiff_p2p_init_local",
     "lowdiff_p2p_destroy", "lowdiff_p2p_slot", "lowdiff_p2p_allgather_sparse", "lowdiff_p2p_status",
-    "lowdiff_batch_merge_ex", "lowdiff_plan_init", "lowdiff_plan_record_due",
+    "lowdiff_batch_merge_ex", "lowdiff_plan_init", "lowdiff_plan_record_due", "lowdiff_replay_check",
 ]
 
 _lib = None
@@ -160,6 +160,7 @@ def lib() -> C.CDLL:
         "lowdiff_p2p_status": ([vp], i32),
         "lowdiff_plan_init": ([vp, u64, f64, C.c_uint32, C.c_uint32, i32, i32, i32, i32], i32),
         "lowdiff_plan_record_due": ([vp, u64, vp, vp, vp], i32),
+        "lowdiff_replay_check": ([vp, vp], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -197,7 +198,9 @@ def workspace(nbytes: int, device, tag: str = "ws") -> torch.Tensor:
     key = (str(d), tag)
     buf = _ws_cache.get(key)
     if buf is None or buf.numel() < nbytes:
-        buf = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=device)
+        # zeroed once (the compress threshold state reads a fresh workspace as cold either way;
+        # zeroing keeps compute-sanitizer initcheck quiet about that intended read)
+        buf = torch.zeros(max(nbytes, 256), dtype=torch.uint8, device=device)
         _ws_cache[key] = buf
     return buf
 
@@ -592,10 +595,12 @@ def _replay_args(state: dict, opt: dict, records):
     return o, st, views, R, keep
 
 
-def replay(state: dict, opt: dict, records, ws=None, stream=None) -> dict:
+def replay(state: dict, opt: dict, records, ws=None, stream=None, check: bool = True) -> dict:
     """Recovery (Alg.1 lines 16-24): replay records [(d_record uint8 CUDA tensor, h_head host bytes)]
     onto the state {x, m, v (fp32 CUDA), x_bf16 (optional), n, lo, hi, t, adam_step,
-    momentum_initialized}; device arrays are updated in place, counters in the dict."""
+    momentum_initialized}; device arrays are updated in place, counters in the dict.
+    check: synchronize and raise ECORRUPT if a record body failed the device validation (the state
+    is then untouched); False leaves that to a later replay_check(ws)."""
     o, st, views, R, keep = _replay_args(state, opt, records)
     b = C.c_uint64()
     _check(lib().lowdiff_replay_workspace_size(C.byref(st), views, R, C.byref(b)), "replay_workspace_size")
@@ -605,7 +610,18 @@ def replay(state: dict, opt: dict, records, ws=None, stream=None) -> dict:
                                 _stream(stream)), "replay")
     state["t"], state["adam_step"] = st.t, st.adam_step
     state["momentum_initialized"] = st.momentum_initialized
+    if check and R:
+        replay_check(ws, stream)
     return state
+
+
+def replay_check(ws=None, stream=None):
+    """lowdiff_replay_check: ECORRUPT if the last replay with this workspace rejected a record body."""
+    if ws is None:
+        ws = _ws_cache.get((f"cuda:{torch.cuda.current_device()}", "replay"))
+        if ws is None:
+            return
+    _check(lib().lowdiff_replay_check(_cuda(ws, "ws"), _stream(stream)), "replay_check")
 
 
 def update(state: dict, opt: dict, g_t, ws=None, stream=None) -> dict:

@@ -446,6 +446,7 @@ static lowdiff_status build_recinfo(const lowdiff_state* st, const lowdiff_opt* 
       r.off_val = r.off_it + pad16(h.nent);
     }
     r.h_lr = lr;
+    r.h_head_bytes = recs[q].h_head;
   }
   return LOWDIFF_OK;
 }
@@ -485,6 +486,11 @@ lowdiff_status lowdiff_replay(lowdiff_state* st, const lowdiff_opt* opt, const l
   if (!ws || !aligned16(ws) || ws_bytes < replay_ws_bytes(st->hi - st->lo, R.data(), nrec))
     return fail(LOWDIFF_EWORKSPACE, "replay: workspace too small");
   return replay_run(st, opt, R.data(), nrec, ws, (cudaStream_t)stream);
+}
+
+lowdiff_status lowdiff_replay_check(const void* ws, lowdiff_stream_t stream) {
+  if (!ws) return fail(LOWDIFF_EINVAL, "replay_check: null workspace");
+  return replay_check(ws, (cudaStream_t)stream);
 }
 
 lowdiff_status lowdiff_update_workspace_size(const lowdiff_state* st, uint64_t* bytes) {

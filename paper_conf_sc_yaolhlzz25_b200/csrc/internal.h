@@ -75,6 +75,7 @@ struct RecInfo {            // parsed on the host from the record header
   uint64_t nnz, nent;
   uint64_t off_lr, off_idx, off_val, off_off, off_it;   // section byte offsets
   const float* h_lr;        // host lr[B]
+  const void* h_head_bytes = nullptr;   // host copy of the 80-byte header (validated against the device)
   // live update (lowdiff_update): a bare (idx, val) list whose length lives on the device; then
   // d == nullptr, mode == SUM, B == 1 and nnz is the host upper bound (cap)
   const uint32_t* live_idx = nullptr;
@@ -84,6 +85,7 @@ struct RecInfo {            // parsed on the host from the record header
 uint64_t replay_ws_bytes(uint64_t len, const RecInfo* recs, uint32_t nrec);
 lowdiff_status replay_run(lowdiff_state* st, const lowdiff_opt* o, const RecInfo* recs,
                           uint32_t nrec, void* ws, cudaStream_t s);
+lowdiff_status replay_check(const void* ws, cudaStream_t s);
 uint64_t replay_parallel_ws_bytes(uint32_t nrec, uint64_t entries, uint64_t lo, uint64_t hi);
 lowdiff_status replay_parallel_run(lowdiff_state* st, const RecInfo* recs, uint32_t nrec, void* ws,
                                    cudaStream_t s);

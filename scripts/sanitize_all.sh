@@ -8,7 +8,7 @@ for tool in memcheck racecheck synccheck initcheck; do
     extra=""
     [ $tool = memcheck ] && extra="--leak-check no"
     LOWDIFF_FAST_SELECT=$fast timeout 1200 /usr/local/cuda/bin/compute-sanitizer --tool $tool $extra \
-      --print-limit 20 python scripts/sanitize_path.py \
+      --print-limit 200 python scripts/sanitize_path.py \
       > gpurun_out/sanitize_${tool}_fast${fast}.log 2>&1
     echo "$tool fast=$fast rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY' gpurun_out/sanitize_${tool}_fast${fast}.log | tail -1)"
   done

@@ -20,7 +20,7 @@ cfg = CONFIGS[1]
 n, k, B = cfg.n, cfg.k, 4
 sig = segment_sigmas(cfg, dev)
 r = torch.zeros(n, device=dev)
-ws = torch.empty(ld.compress_workspace_size(n, k), dtype=torch.uint8, device=dev)
+ws = torch.zeros(ld.compress_workspace_size(n, k), dtype=torch.uint8, device=dev)
 ring = []
 for t in range(6):                                   # cold (rescan), then warm calls
     g = gradient(cfg, 0, t, dev, sigmas=sig)
@@ -30,7 +30,7 @@ for t in range(6):                                   # cold (rescan), then warm 
 print("compress paths", ld.compress_counters(ws=ws))
 # a larger k so the grid select (fast path) runs instead of the one-CTA select
 k2 = 20_000
-ws2 = torch.empty(ld.compress_workspace_size(n, k2), dtype=torch.uint8, device=dev)
+ws2 = torch.zeros(ld.compress_workspace_size(n, k2), dtype=torch.uint8, device=dev)
 r2 = torch.zeros(n, device=dev)
 for t in range(4):
     ld.compress(gradient(cfg, 0, t, dev, sigmas=sig), r2, k2, ws=ws2)
