@@ -135,6 +135,36 @@ def oracle_all_cores(cfg, n_s: int, grads, procs: int) -> dict:
             "wall_s": wall}
 
 
+def max_over_ranks(ms: float, world: int) -> float:
+    """The step time of the whole job: the slowest rank's device time (all_reduce MAX over the
+    host process group; identity at world 1)."""
+    if world <= 1:
+        return ms
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([ms], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def rank_table(world: int, rank: int, local: int, nbytes: int, nnz: int) -> list | None:
+    """Per-rank device id, PCI bus id and shard record size, gathered to rank 0 (evidence that
+    every rank ran on its own GPU, and the shard skew of SURVEY §8(e))."""
+    import torch
+    pci = None
+    try:
+        pci = torch.cuda.get_device_properties(local).pci_bus_id
+    except Exception:
+        pass
+    mine = {"rank": rank, "device": local, "pci_bus_id": pci, "record_bytes": int(nbytes), "nnz": int(nnz)}
+    if world <= 1:
+        return [mine]
+    import torch.distributed as dist
+    out = [None] * world
+    dist.all_gather_object(out, mine)
+    return out if rank == 0 else None
+
+
 def chain_records(cfg) -> int:
     """Records per step: the config's replay chain of K differentials is K/B batch records."""
     return max(1, cfg.K // cfg.B)
@@ -256,7 +286,21 @@ def run_ours(args, cfg):
         except ld.LowDiffError as e:                    # e.g. no IPC / peer access between the GPUs
             sync_note = f"p2p unavailable ({e}); ncclAllGather + coalesce"
             print(sync_note, file=sys.stderr)
-    comm = ld.Comm(P, rank) if P > 1 and p2p is None else None
+    # N > 1: the NCCL communicator always exists (the baseline Sync route; with the fused P2P Sync
+    # as the default it is timed as a second arm below), so every multi-GPU run shows NCCL
+    comm, nccl_note = None, None
+    if P > 1:
+        try:
+            comm = ld.Comm(P, rank)
+        except ld.LowDiffError as e:                    # e.g. several ranks sharing one GPU (liveness runs)
+            if p2p is None:
+                raise
+            nccl_note = f"NCCL communicator unavailable ({e}); P2P Sync only"
+            print(nccl_note, file=sys.stderr)
+    if P > 1:
+        print(f"lowdiff rank {rank}/{P}: cuda:{local} ({torch.cuda.get_device_name(local)}), NCCL communicator "
+              f"{'+ P2P exchange windows' if p2p is not None else 'only'}" if comm is not None else
+              f"lowdiff rank {rank}/{P}: cuda:{local}, P2P exchange windows", file=sys.stderr, flush=True)
 
     # ---- resident inputs: B gradients (seeded, per rank), residual, full-checkpoint shard ----
     sig = segment_sigmas(cfg, dev)
@@ -304,6 +348,8 @@ def run_ours(args, cfg):
     ev_copy = [torch.cuda.Event() for _ in range(2)]
     ev_free = [torch.cuda.Event() for _ in range(2)]
 
+    use_p2p = [p2p is not None]                       # the Sync route of the build phase
+
     def build_phase(h2d=None):
         """B iterations of compress -> sparse all-gather + coalesce of this rank's shard -> ring.
         e2e (h2d given): iteration j's gradient is copied from pinned host memory on a copy stream
@@ -324,7 +370,8 @@ def run_ours(args, cfg):
                 g = h2d[0][d]
             else:
                 g = grads[j % len(grads)]
-            dst = p2p.slot() if p2p is not None else pairs   # p2p: compress straight into the window
+            pp = p2p if use_p2p[0] else None
+            dst = pp.slot() if pp is not None else pairs     # p2p: compress straight into the window
             if zero_copy:
                 dst = slots[j]
             ld.compress(g, r, k, vdt=cfg.vdt, pairs=dst, ws=cws)
@@ -332,8 +379,8 @@ def run_ours(args, cfg):
                 ev_free[d].record(cs)
             if zero_copy:
                 pass                                    # the slot already holds G~_t
-            elif p2p is not None:
-                p2p.allgather_sparse(dst, lo, hi, True, *ring[j])
+            elif pp is not None:
+                pp.allgather_sparse(dst, lo, hi, True, *ring[j])
             else:
                 ld.allgather_sparse(comm, pairs, k, cfg.vdt, lo, hi, True, *ring[j])
         if h2d is not None:
@@ -385,11 +432,8 @@ def run_ours(args, cfg):
             nb = step(**kw)
         e1.record()
         torch.cuda.synchronize()
-        ms = e0.elapsed_time(e1)
+        ms = max_over_ranks(e0.elapsed_time(e1), world)
         if world > 1:
-            t = torch.tensor([ms], dtype=torch.float64)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            ms = float(t.item())
             dist.barrier()
         return ms, nb
 
@@ -445,6 +489,22 @@ def run_ours(args, cfg):
                                              "replay_dense", "replay_sparse")}
     ms_step = ms / args.steps
     value = P * R * B * n * gsz / (ms_step * 1e-3) / 1e9
+    # ---- N > 1: the same steps with the baseline Sync (ncclAllGather + coalesce) as a second arm ----
+    sync_arms = None
+    if P > 1:
+        sync_arms = {("p2p" if use_p2p[0] else "nccl"): ms_step}
+        if p2p is not None and comm is not None:
+            use_p2p[0] = False
+            g_nccl, _ = capture()
+            step(graph=g_nccl) if g_nccl is not None else step()
+            ms_n, _ = timed(args.steps, graph=g_nccl) if g_nccl is not None else timed(args.steps)
+            sync_arms["nccl"] = ms_n / args.steps
+            use_p2p[0] = True
+        sync_arms["unit"] = "ms per step (max over ranks)"
+        if nccl_note:
+            sync_arms["note"] = nccl_note
+    nnz_rank = int(np.frombuffer(heads[0].numpy().tobytes()[:80], dtype=np.uint64)[7]) if R else 0
+    ranks = rank_table(world, rank, local, sum(rec_nb), nnz_rank)
 
     # ---- roofline of the dominant kernel (measured live over the timed region) ----
     peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
@@ -629,6 +689,10 @@ def run_ours(args, cfg):
                                                "with the records copied H2D from pinned memory first "
                                                "(profiled pass, CUDA events)",
                            "record_bytes": int(rec_bytes),
+                           "ranks": ranks,
+                           "shard_skew": (max(x["record_bytes"] for x in ranks) /
+                                          (sum(x["record_bytes"] for x in ranks) / len(ranks))) if ranks else None,
+                           "sync_arms": sync_arms,
                            "compress_paths": paths},
                 "timing": {"build_phase": "one CUDA graph per step" if graph is not None else "eager launches",
                            "profiled_ms_per_step": pms / args.steps,

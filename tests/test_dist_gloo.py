@@ -80,6 +80,16 @@ def _worker(rank, world, port, q):
         assert np.array_equal(np.concatenate([np.array(x[0], np.uint32) for x in recs]), full["idx"])
         assert np.array_equal(np.concatenate([np.array(x[1], np.uint32) for x in recs]),
                               full["val"].view(np.uint32))
+        # 4. bench.py's multi-rank plumbing: the job's step time is the slowest rank's, and rank 0
+        #    gathers every rank's device / shard-record evidence (the driver reads both)
+        import bench
+        assert bench.max_over_ranks(10.0 + 5.0 * rank, world) == 10.0 + 5.0 * (world - 1)
+        table = bench.rank_table(world, rank, rank, 1000 * (rank + 1), 7 * (rank + 1))
+        if rank == 0:
+            assert [row["rank"] for row in table] == list(range(world))
+            assert [row["record_bytes"] for row in table] == [1000 * (p + 1) for p in range(world)]
+        else:
+            assert table is None
         dist.barrier()
         dist.destroy_process_group()
         q.put((rank, "ok"))
