@@ -59,6 +59,7 @@ struct __align__(256) State {
 };
 struct StateKey {
   uint64_t n, k, resid, tag;
+  float band_lo, band_hi;   // the margin controller's target band of first-pass candidates / k
 };
 constexpr float kDeltaInit = 1.0f / 64, kDeltaMin = 1.0f / 8192, kDeltaMax = 0.5f;
 
@@ -169,7 +170,8 @@ __device__ __forceinline__ uint32_t fine_bin(uint32_t key, uint32_t T, uint32_t 
 }
 
 // After the select (one thread): counters, and the margin controller on the first pass's
-// candidate count: fewer than k -> widen, above the capacity -> narrow, else aim at 1.2-3 k.
+// candidate count: fewer than k -> widen, above the capacity -> narrow, else aim at the band
+// (1.05-1.5 k by default: fewer candidates make the select cheaper, scripts/band_sweep.sh).
 __device__ void state_update(State* st, const StateKey& sk, uint64_t k, uint32_t cap, uint32_t cc,
                              uint32_t path, uint32_t kstar, uint64_t nonfinite) {
   const bool warm = state_valid(st, sk);
@@ -181,8 +183,8 @@ __device__ void state_update(State* st, const StateKey& sk, uint64_t k, uint32_t
     float d = st->delta;
     if (cc < k) d = d * 2.0f;
     else if (cc > cap) d = d * 0.5f;
-    else if ((double)cc > 3.0 * (double)k) d = d * 0.75f;
-    else if ((double)cc < 1.2 * (double)k) d = d * 1.5f;
+    else if ((double)cc > (double)sk.band_hi * (double)k) d = d * 0.75f;
+    else if ((double)cc < (double)sk.band_lo * (double)k) d = d * 1.5f;
     st->delta = d < kDeltaMin ? kDeltaMin : (d > kDeltaMax ? kDeltaMax : d);
   }
   st->calls += 1;
@@ -1582,7 +1584,15 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   Ctl* ctl = reinterpret_cast<Ctl*>(w + L.ctl);
   State* st = reinterpret_cast<State*>(w + L.state);
   LD_CUDA(cudaMemsetAsync(w + L.ctl, 0, L.zero_end - L.ctl, s), "memset compress workspace");
-  const StateKey sk{n, k, (uint64_t)(uintptr_t)residual, (uint64_t)(gdt | (vdt << 8))};
+  static float band_lo = 0.f, band_hi = 0.f;
+  if (band_lo == 0.f) {                            // LOWDIFF_CAND_BAND="lo,hi" (experiments)
+    band_lo = 1.05f; band_hi = 1.5f;              // measured: scripts/band_sweep.sh (profiles/r02/band.txt)
+    if (const char* e = getenv("LOWDIFF_CAND_BAND")) {
+      float a = 0.f, b = 0.f;
+      if (sscanf(e, "%f,%f", &a, &b) == 2 && a >= 1.0f && b > a) { band_lo = a; band_hi = b; }
+    }
+  }
+  const StateKey sk{n, k, (uint64_t)(uintptr_t)residual, (uint64_t)(gdt | (vdt << 8)), band_lo, band_hi};
 
   // recovery sample size: >= 512 expected keys above the k-th (S >= 512 n / k: the 2x target is
   // then > 10 sigma of the count above k), >= 64 Ki, power of 2; every micro-chunk when S >= n/2

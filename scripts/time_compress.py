@@ -33,7 +33,7 @@ def loop():
         ld.compress(g, r, cfg.k, vdt=cfg.vdt, pairs=pairs, ws=ws)
 
 
-for _ in range(3):
+for _ in range(6):
     loop()
 torch.cuda.synchronize()
 g = torch.cuda.CUDAGraph()
