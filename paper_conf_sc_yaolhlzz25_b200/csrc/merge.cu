@@ -732,8 +732,18 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
   // list is found first and only it is scanned (batch merge: the lists are the shard's already)
   uint32_t* ebnd = kind == kCoalesce ? reinterpret_cast<uint32_t*>(w + M.ebnd) : nullptr;
   if (ebnd) LD_LAUNCH("starts", s, bounds_kernel, ls.L, 64, 0, ls, lo, hi, ebnd);
-  LD_LAUNCH("starts", s, starts_kernel<kW>, dim3((unsigned)gx, (unsigned)ls.L), kThreads, 0, ls, lo, hi,
-            M.num_w, starts, (const uint32_t*)ebnd);
+  bool al16 = !ebnd;
+  for (int l = 0; l < ls.L && al16; ++l) al16 = (reinterpret_cast<uintptr_t>(ls.list[l].idx) & 15u) == 0;
+  if (al16) {                                      // 16-byte loads, 2 steps in flight
+    uint64_t g4 = (per_list / 4 + 1 + 2 * kThreads - 1) / (2 * kThreads);
+    if (g4 > 8ull * kNumSMs) g4 = 8ull * kNumSMs;
+    if (g4 < 1) g4 = 1;
+    LD_LAUNCH("starts", s, starts4_kernel<kW>, dim3((unsigned)g4, (unsigned)ls.L), kThreads, 0, ls, lo, hi,
+              M.num_w, starts);
+  } else {
+    LD_LAUNCH("starts", s, starts_kernel<kW>, dim3((unsigned)gx, (unsigned)ls.L), kThreads, 0, ls, lo, hi,
+              M.num_w, starts, (const uint32_t*)ebnd);
+  }
 
   // group size: up to kCap/2 entries per group at the average density (power of two); the
   // entries actually present (max_entries is a capacity) make groups smaller than this bound

@@ -57,6 +57,83 @@ __global__ void __launch_bounds__(kThreads) starts_kernel(const __grid_constant_
   }
 }
 
+// The same starts table, 4 entries per thread per step with 16-byte loads and 2 steps in flight
+// (lists whose idx base is 16-byte aligned, no ebnd): the HBM-bound form for long lists (replay
+// records, batch-merge lists). Entry e writes the windows in (win(e-1), win(e)]; e = len writes
+// the tail up to num_w. Long gaps are filled by the whole warp, coalesced.
+template <int W>
+__global__ void __launch_bounds__(kThreads) starts4_kernel(const __grid_constant__ ListSet ls, uint64_t lo,
+                                                           uint64_t hi, uint32_t num_w, uint32_t* starts) {
+  static_assert((W & (W - 1)) == 0, "W is a power of two");
+  constexpr int kLog = __builtin_ctz(W);
+  const int l = blockIdx.y;
+  const uint32_t* idx = ls.list[l].idx;
+  const uint32_t len = (uint32_t)list_len(ls, l);   // < 2^31
+  uint32_t* st = starts + (uint64_t)l * (num_w + 1);
+  const int lane = threadIdx.x & 31;
+  const uint32_t lo32 = (uint32_t)lo, hi32 = (uint32_t)hi;
+  auto win_of = [&](uint32_t i) -> int32_t {         // window of an index value (32-bit: n < 2^31)
+    if (i < lo32) return -1;
+    if (i >= hi32) return (int32_t)num_w;
+    return (int32_t)((i - lo32) >> kLog);
+  };
+  const uint32_t nq = len / 4 + 1;                 // quads; the last (partial) quad carries e = len
+  const uint32_t stride = gridDim.x * kThreads;
+  for (uint32_t q0 = blockIdx.x * kThreads + (threadIdx.x & ~31u); q0 < nq; q0 += 2 * stride) {
+    uint4 v[2];
+    uint32_t before[2];
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {                  // both steps' loads first
+      const uint32_t q = q0 + h * stride + lane;
+      const uint32_t e = 4 * q;
+      v[h] = make_uint4(0u, 0u, 0u, 0u);
+      if (q < nq) {
+        if (e + 4 <= len) {
+          v[h] = *reinterpret_cast<const uint4*>(idx + e);
+        } else {
+          uint32_t t[4] = {0u, 0u, 0u, 0u};
+          for (uint32_t j = 0; j < 4; ++j) if (e + j < len) t[j] = idx[e + j];
+          v[h] = make_uint4(t[0], t[1], t[2], t[3]);
+        }
+      }
+      before[h] = (lane == 0 && e > 0 && q < nq) ? idx[e - 1] : 0u;
+    }
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      if (q0 + h * stride >= nq) break;            // warp-uniform
+      const uint32_t q = q0 + h * stride + lane;
+      const uint32_t e = 4 * q;
+      const uint32_t up = __shfl_up_sync(0xFFFFFFFFu, v[h].w, 1);
+      const uint32_t iv[4] = {v[h].x, v[h].y, v[h].z, v[h].w};
+      int32_t wv[5];                               // windows of entries e-1 .. e+3 (num_w at e+j = len)
+      wv[0] = (e == 0 || q >= nq) ? -1 : win_of(lane == 0 ? before[h] : up);
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        wv[j + 1] = (q >= nq || e + j > len) ? wv[j] : (e + j == len ? (int32_t)num_w : win_of(iv[j]));
+      bool longr = false;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        if (wv[j + 1] - wv[j] > 8) longr = true;
+        else for (int32_t w = wv[j] + 1; w <= wv[j + 1]; ++w) st[w] = e + j;
+      }
+      uint32_t lm = __ballot_sync(0xFFFFFFFFu, longr);
+      while (lm) {                                 // long gaps (rare): the whole warp fills them
+        const int src = __ffs(lm) - 1;
+        lm &= lm - 1;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const int32_t from = __shfl_sync(0xFFFFFFFFu, wv[j], src) + 1;
+          const int32_t to = __shfl_sync(0xFFFFFFFFu, wv[j + 1], src);
+          if (to - from + 1 > 8) {                 // (uniform) this entry's gap
+            const uint32_t ee = __shfl_sync(0xFFFFFFFFu, e, src) + j;
+            for (int32_t w = from + lane; w <= to; w += 32) st[w] = ee;
+          }
+        }
+      }
+    }
+  }
+}
+
 // ebnd[2l] / ebnd[2l+1] = first position of list l with idx >= lo / idx >= hi (lists strictly
 // ascending). One block of 64 threads per list, one warp per bound: a 32-ary search, each round a
 // single coalesced probe of 32 positions (about 5 dependent rounds for a list of 3.4 M entries).
