@@ -334,7 +334,7 @@ def run_ours(args, cfg):
         slots = [torch.empty(ld.pairs_bytes(k, cfg.vdt), dtype=torch.uint8, device=dev) for _ in range(B)]
         d_k = torch.full((1,), k, dtype=torch.int64, device=dev)
         ring = [ld.pairs_views(sl, k, cfg.vdt) + (d_k,) for sl in slots]
-    rec_cap = ld.record_max_bytes(cfg.merge, B, B * cap)
+    rec_cap = ld.record_max_bytes(cfg.merge, B, B * cap, lo, hi)
     R = chain_records(cfg)                              # batch records per step (replay chain K = R*B)
     records = [torch.empty(rec_cap, dtype=torch.uint8, device=dev) for _ in range(R)]
     d_bytes = torch.zeros(1, dtype=torch.int64, device=dev)

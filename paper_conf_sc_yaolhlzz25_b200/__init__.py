@@ -91,6 +91,7 @@ EXPORTS = [
     "lowdiff_p2p_window_bytes", "lowdiff_p2p_export_handle", "lowdiff_p2p_init", "lowdiff_p2p_init_local",
     "lowdiff_p2p_destroy", "lowdiff_p2p_slot", "lowdiff_p2p_allgather_sparse", "lowdiff_p2p_status",
     "lowdiff_batch_merge_ex", "lowdiff_plan_init", "lowdiff_plan_record_due", "lowdiff_replay_check",
+    "lowdiff_record_max_bytes_shard",
 ]
 
 _lib = None
@@ -161,6 +162,7 @@ def lib() -> C.CDLL:
         "lowdiff_plan_init": ([vp, u64, f64, C.c_uint32, C.c_uint32, i32, i32, i32, i32], i32),
         "lowdiff_plan_record_due": ([vp, u64, vp, vp, vp], i32),
         "lowdiff_replay_check": ([vp, vp], i32),
+        "lowdiff_record_max_bytes_shard": ([i32, C.c_uint32, u64, u64, u64], u64),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -273,7 +275,10 @@ def record_size(mode, B: int, nnz: int, nent: int) -> int:
     return int(lib().lowdiff_record_size(_MODE[mode], B, nnz, nent))
 
 
-def record_max_bytes(mode, B: int, max_entries: int) -> int:
+def record_max_bytes(mode, B: int, max_entries: int, lo: int | None = None, hi: int | None = None) -> int:
+    """Upper bound of a record's bytes; with the shard [lo, hi) its unique indices are bounded too."""
+    if lo is not None and hi is not None:
+        return int(lib().lowdiff_record_max_bytes_shard(_MODE[mode], B, max_entries, lo, hi))
     return int(lib().lowdiff_record_max_bytes(_MODE[mode], B, max_entries))
 
 

@@ -312,6 +312,12 @@ uint64_t lowdiff_record_max_bytes(lowdiff_merge_mode mode, uint32_t B, uint64_t 
   return lowdiff_record_size(mode, B, max_entries, max_entries);
 }
 
+uint64_t lowdiff_record_max_bytes_shard(lowdiff_merge_mode mode, uint32_t B, uint64_t max_entries, uint64_t lo,
+                                        uint64_t hi) {
+  const uint64_t u = hi > lo && hi - lo < max_entries ? hi - lo : max_entries;   // unique indices <= shard
+  return lowdiff_record_size(mode, B, u, max_entries);
+}
+
 lowdiff_status lowdiff_batch_merge_workspace_size(uint32_t B, uint64_t max_entries, uint64_t lo, uint64_t hi,
                                                   uint64_t* bytes) {
   if (!bytes || B == 0 || B > 255 || lo >= hi || hi > (1ull << 31) || max_entries >= (1ull << 31))

@@ -91,7 +91,7 @@ class LowDiffLoop:
         self.pairs = torch.empty(pairs_bytes(self.k), dtype=torch.uint8, device=dev)
         if not checkpoint:
             return
-        self.rec_cap = record_max_bytes("stack", B, max(B * self.cap, 1))
+        self.rec_cap = record_max_bytes("stack", B, max(B * self.cap, 1), self.lo, self.hi)
         # two device record buffers: one being merged while the other is staged
         self.drec = [{"buf": torch.empty(self.rec_cap, dtype=torch.uint8, device=dev),
                       "nb": torch.zeros(1, dtype=torch.int64, device=dev),

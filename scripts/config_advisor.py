@@ -5,9 +5,11 @@ line and the job's own parameters, through the library's lowdiff_optimal_config.
     python scripts/config_advisor.py bench.json --iter-ms 350 --mtbf-h 24 --write-gbs 2 \
         --gpus 8 --hours 72 --load-full-s 60
 
-R_D (time to merge one differential) is taken from the bench line's replay (replay ms per step /
-replayed iterations per step); S from the full checkpoint the bench replays onto (x, m, v fp32 of
-the shard, times P ranks). Every time is converted to training iterations (reading #29).
+R_D is the time to merge (replay) ONE batched differential checkpoint onto the full one: Eq. 3 counts
+1/(f b) batched records per chain, so R_D is the bench line's replay time per step
+divided by the records per step (a STACK record of B iterations replays B optimizer steps); S is
+the full checkpoint the bench replays onto (x, m, v fp32 of the shard, times P ranks). Every time is
+converted to training iterations (reading #29).
 """
 import argparse
 import json
@@ -30,8 +32,8 @@ def main():
     import paper_conf_sc_yaolhlzz25_b200 as ld
     d = json.loads(open(a.bench_json).read().strip().splitlines()[-1])
     cfg = d["config"]
-    k_iters = cfg["B"] * cfg.get("batches_per_step", 1)
-    rd_ms = d["kernels"].get("replay_dense", d["kernels"].get("replay_sparse"))["ms_per_step"] / k_iters
+    records = cfg.get("batches_per_step", 1)
+    rd_ms = d["kernels"].get("replay_dense", d["kernels"].get("replay_sparse"))["ms_per_step"] / records
     state_bytes = {"sgd": 4, "momentum": 8, "adam": 12}[cfg["replay"].split(",")[0]] * cfg["n"]
     it_s = a.iter_ms * 1e-3
     model = {"N": a.gpus, "M": a.mtbf_h * 3600 / it_s, "W": a.write_gbs * 1e9 * it_s, "S": state_bytes,

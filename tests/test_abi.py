@@ -55,6 +55,19 @@ def test_host_helpers_match_definitions():
             assert ld.record_size(mode, B, nnz, nent) == oracle.record_size(om, B, nnz, nent)
 
 
+def test_record_max_bytes_shard_bound():
+    """A shard's record has at most hi - lo unique indices (bound the record buffers by
+    min(B cap, hi - lo)); the entries stay bounded by max_entries."""
+    for mode in ("sum", "stack"):
+        for B, me, lo, hi in ((32, 400_000_000, 0, 194_701_400), (8, 1000, 10, 5000), (4, 10, 0, 1_000_000)):
+            u = min(me, hi - lo)
+            assert ld.record_max_bytes(mode, B, me, lo, hi) == ld.record_size(mode, B, u, me if mode == "stack" else u)
+            assert ld.record_max_bytes(mode, B, me, lo, hi) <= ld.record_max_bytes(mode, B, me)
+    # C5 shard, STACK, B = 32 differentials of ~12.5 M entries
+    assert ld.record_max_bytes("stack", 32, 32 * 12_460_888, 0, 194_701_400) < 3.7e9 < \
+        ld.record_max_bytes("stack", 32, 32 * 12_460_888)
+
+
 def test_p2p_window_layout():
     """Exchange window of the fused Sync (include/lowdiff.h (2')): u64 ready[P] | u64 done[P] |
     u64 epoch, padded to 256 B, then two 256-B aligned slots of one packed pairs buffer each."""
