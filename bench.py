@@ -403,6 +403,8 @@ def run_ours(args, cfg):
     def recovery_phase():
         """Load(C^F) + replay of the step's chain of R records (K = R*B iterations)."""
         main.synchronize()                              # the replay call reads the staged headers
+        if os.environ.get("LOWDIFF_BENCH_SERIAL_STAGE"):  # experiment: staging not overlapped with replay
+            copy_stream.synchronize()
         state["t"] = t_iter[0] - R * B                  # the checkpoint is stamped at the chain start
         state["adam_step"] = ck["adam_step"]
         state["momentum_initialized"] = ck["momentum_initialized"]

@@ -75,4 +75,27 @@ __device__ inline uint64_t block_exclusive_scan(uint64_t x, uint64_t* smem, uint
   return warp_off + incl - x;
 }
 
+// The same for a block of NT threads (NT % 32 == 0, NT <= 1024); `smem` holds >= NT/32 u64.
+template <int NT>
+__device__ inline uint64_t block_exclusive_scan_n(uint64_t x, uint64_t* smem, uint64_t* total) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint64_t incl = x;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint64_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+    if (lane >= o) incl += y;
+  }
+  if (lane == 31) smem[warp] = incl;
+  __syncthreads();
+  uint64_t warp_off = 0, tot = 0;
+  for (int w = 0; w < NT / 32; ++w) {
+    uint64_t t = smem[w];
+    if (w < warp) warp_off += t;
+    tot += t;
+  }
+  __syncthreads();
+  *total = tot;
+  return warp_off + incl - x;
+}
+
 }  // namespace lowdiff

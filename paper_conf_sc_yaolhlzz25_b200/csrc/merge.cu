@@ -91,60 +91,56 @@ __device__ __forceinline__ float list_val(const ListSet& ls, int l, uint64_t e) 
 // items[i] = (first fine window, number of fine windows).
 __global__ void __launch_bounds__(kPlanThreads) plan_kernel(int L, const uint32_t* __restrict__ starts,
                                                             uint32_t num_w, uint32_t G, uint32_t sparse_max,
-                                                            int keep_groups, MCtl* ctl, uint2* __restrict__ items) {
-  __shared__ uint32_t s_warp[kPlanThreads / 32];
-  __shared__ uint32_t s_carry;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+                                                            int keep_groups, MCtl* ctl, uint2* __restrict__ items,
+                                                            uint32_t* __restrict__ gcnt) {
+  __shared__ uint64_t s_scan[kPlanThreads / 32];
+  const int tid = threadIdx.x;
   const uint32_t num_g = (num_w + G - 1) / G;
-  if (tid == 0) s_carry = 0;
+  if (keep_groups) {                               // bitmap-sized groups stay whole: item g = group g
+    for (uint32_t g = tid; g < num_g; g += kPlanThreads)
+      items[g] = make_uint2(g * G, (g * G + G < num_w ? G : num_w - g * G));
+    if (tid == 0) ctl->num_items = num_g;
+    return;
+  }
+  // per group (block-strided: every thread's loads in flight at once) the entry count decides
+  // whole / split into windows -> gcnt; then each thread sums a contiguous chunk of gcnt, one block
+  // scan places every item (index order)
+  auto count = [&](uint32_t g) -> uint32_t {
+    const uint32_t fs = g * G, fe = fs + G < num_w ? fs + G : num_w;
+    uint64_t e = 0;
+    int l = 0;
+    for (; l + 4 <= L; l += 4) {                   // 8 independent loads in flight
+      uint32_t a2[4], b2[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint32_t* st = starts + (uint64_t)(l + q) * (num_w + 1);
+        a2[q] = st[fe]; b2[q] = st[fs];
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) e += a2[q] - b2[q];
+    }
+    for (; l < L; ++l) {
+      const uint32_t* st = starts + (uint64_t)l * (num_w + 1);
+      e += st[fe] - st[fs];
+    }
+    return (e <= (uint64_t)sparse_max || fe - fs == 1) ? 1u : fe - fs;
+  };
+  for (uint32_t g = tid; g < num_g; g += kPlanThreads) gcnt[g] = count(g);
   __syncthreads();
-  for (uint32_t g0 = 0; g0 < num_g; g0 += kPlanThreads) {
-    const uint32_t g = g0 + tid;
-    uint32_t fs = 0, fe = 0, cnt = 0;
-    if (g < num_g) {
-      fs = g * G;
-      fe = fs + G < num_w ? fs + G : num_w;
-      uint64_t e = 0;
-      int l = 0;
-      for (; l + 4 <= L; l += 4) {                   // 8 independent loads in flight
-        uint32_t a[4], b[4];
-#pragma unroll
-        for (int q = 0; q < 4; ++q) {
-          const uint32_t* st = starts + (uint64_t)(l + q) * (num_w + 1);
-          a[q] = st[fe]; b[q] = st[fs];
-        }
-#pragma unroll
-        for (int q = 0; q < 4; ++q) e += a[q] - b[q];
-      }
-      for (; l < L; ++l) {
-        const uint32_t* st = starts + (uint64_t)l * (num_w + 1);
-        e += st[fe] - st[fs];
-      }
-      // keep_groups: bitmap-sized groups stay whole (the bitmap path takes any entry count)
-      cnt = (keep_groups || e <= (uint64_t)sparse_max || fe - fs == 1) ? 1u : fe - fs;
-    }
-    uint32_t incl = cnt;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
-      if (lane >= o) incl += y;
-    }
-    if (lane == 31) s_warp[warp] = incl;
-    __syncthreads();
-    uint32_t off = s_carry, tot = 0;
-    for (int w = 0; w < kPlanThreads / 32; ++w) {
-      if (w < warp) off += s_warp[w];
-      tot += s_warp[w];
-    }
-    off += incl - cnt;
+  const uint32_t per = (num_g + kPlanThreads - 1) / kPlanThreads;
+  const uint32_t g0 = tid * per, g1 = g0 + per < num_g ? g0 + per : num_g;
+  uint32_t mine = 0;
+  for (uint32_t g = g0; g < g1; ++g) mine += gcnt[g];
+  uint64_t tot;
+  uint32_t off = (uint32_t)block_exclusive_scan_n<kPlanThreads>(mine, s_scan, &tot);
+  for (uint32_t g = g0; g < g1; ++g) {
+    const uint32_t cnt = gcnt[g], fs = g * G, fe = fs + G < num_w ? fs + G : num_w;
     if (cnt == 1) items[off] = make_uint2(fs, fe - fs);
     else
-      for (uint32_t s = 0; s < cnt; ++s) items[off + s] = make_uint2(fs + s, 1u);
-    __syncthreads();
-    if (tid == 0) s_carry += tot;
-    __syncthreads();
+      for (uint32_t q = 0; q < cnt; ++q) items[off + q] = make_uint2(fs + q, 1u);
+    off += cnt;
   }
-  if (tid == 0) ctl->num_items = s_carry;
+  if (tid == 0) ctl->num_items = (uint32_t)tot;
 }
 
 // ---- K2b: item merge ------------------------------------------------------------------------------
@@ -236,10 +232,18 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
       //      and the first entry of a slot (rank 0) writes the unique head. No sorting.
       for (uint32_t j = tid; j < (uint32_t)L * NW; j += kThreads) sm.b.bm[j] = 0;
       __syncthreads();
-      for (uint32_t x = tid; x < E; x += kThreads) {
-        const int a = list_of(x);
-        const uint32_t slot = ls.list[a].idx[s_beg[a] + (x - s_off[a])] - (uint32_t)w0;
-        atomicOr(&sm.b.bm[a * NW + (slot >> 5)], 1u << (slot & 31));
+      for (uint32_t x0 = tid; x0 < E; x0 += 4 * kThreads) {   // 4 entries' loads in flight
+        int aa[4];
+        uint32_t sl[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const uint32_t x = x0 + u * kThreads;
+          aa[u] = x < E ? list_of(x) : 0;
+          sl[u] = x < E ? ls.list[aa[u]].idx[s_beg[aa[u]] + (x - s_off[aa[u]])] - (uint32_t)w0 : 0xFFFFFFFFu;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          if (sl[u] != 0xFFFFFFFFu) atomicOr(&sm.b.bm[aa[u] * NW + (sl[u] >> 5)], 1u << (sl[u] & 31));
       }
       __syncthreads();
       // each thread owns q consecutive words: their counts, a block scan, then the per-word prefix
@@ -263,10 +267,23 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
         run += ((uint64_t)__popc(sm.b.orw[wd]) << 32) | c;
       }
       __syncthreads();
-      for (uint32_t x = tid; x < E; x += kThreads) {
-        const int a = list_of(x);
-        const uint64_t e = s_beg[a] + (x - s_off[a]);
-        const uint32_t slot = ls.list[a].idx[e] - (uint32_t)w0;
+      for (uint32_t x0 = tid; x0 < E; x0 += 4 * kThreads) {   // 4 entries' (idx, val) loads in flight
+        int aa[4];
+        uint32_t sl[4];
+        float vv[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const uint32_t x = x0 + u * kThreads;
+          aa[u] = x < E ? list_of(x) : 0;
+          const uint64_t e = s_beg[aa[u]] + (x - s_off[aa[u]]);
+          sl[u] = x < E ? ls.list[aa[u]].idx[e] - (uint32_t)w0 : 0xFFFFFFFFu;
+          vv[u] = x < E ? list_val<BF16>(ls, aa[u], e) : 0.f;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+        if (sl[u] == 0xFFFFFFFFu) break;
+        const int a = aa[u];
+        const uint32_t slot = sl[u];
         const uint32_t wd = slot >> 5, bit = 1u << (slot & 31), below = bit - 1u;
         uint32_t cb = 0, rank = 0;
         for (int l = 0; l < L; ++l) {
@@ -277,11 +294,12 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
         const uint64_t pw = sm.b.wpre[wd];
         const uint32_t pos = e0 + (uint32_t)pw + cb + rank;
         out_it[pos] = (uint8_t)a;
-        out_ent[pos] = list_val<BF16>(ls, a, e);
+        out_ent[pos] = vv[u];
         if (rank == 0) {
-          const uint32_t u = e0 + (uint32_t)(pw >> 32) + __popc(sm.b.orw[wd] & below);
-          stg_idx[u] = (uint32_t)(w0 + slot);
-          stg_val[u] = pos;                        // off[] = the head's entry position
+          const uint32_t uu = e0 + (uint32_t)(pw >> 32) + __popc(sm.b.orw[wd] & below);
+          stg_idx[uu] = (uint32_t)(w0 + slot);
+          stg_val[uu] = pos;                       // off[] = the head's entry position
+        }
         }
       }
       tot >>= 32;                                  // unique slots of the item
@@ -442,32 +460,29 @@ __global__ void __launch_bounds__(kPlanThreads) ucount_scan_kernel(const __grid_
                                                                    MCtl* ctl, const uint32_t* __restrict__ ucnt,
                                                                    uint32_t* __restrict__ upre,
                                                                    uint64_t* d_out_nnz) {
-  __shared__ uint32_t s_warp[kPlanThreads / 32];
-  __shared__ uint32_t s_carry;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  __shared__ uint64_t s_scan[kPlanThreads / 32];
+  const int tid = threadIdx.x;
   const uint32_t num_items = ctl->num_items;
-  if (tid == 0) s_carry = 0;
-  __syncthreads();
-  for (uint32_t i0 = 0; i0 < num_items; i0 += kPlanThreads) {
-    const uint32_t i = i0 + tid;
-    const uint32_t c = i < num_items ? ucnt[i] : 0u;
-    uint32_t incl = c;
+  // each thread a contiguous chunk of items (4 loads in flight), one block scan of the chunk sums
+  const uint32_t per = (num_items + kPlanThreads - 1) / kPlanThreads;
+  const uint32_t i0 = tid * per, i1 = i0 + per < num_items ? i0 + per : num_items;
+  uint32_t mine = 0;
+  for (uint32_t i = i0; i < i1; i += 4) {
+    uint32_t v[4];
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
-      if (lane >= o) incl += y;
-    }
-    if (lane == 31) s_warp[warp] = incl;
-    __syncthreads();
-    uint32_t off = s_carry, tot = 0;
-    for (int w = 0; w < kPlanThreads / 32; ++w) {
-      if (w < warp) off += s_warp[w];
-      tot += s_warp[w];
-    }
-    if (i < num_items) upre[i] = off + incl - c;
-    __syncthreads();
-    if (tid == 0) s_carry += tot;
-    __syncthreads();
+    for (int q = 0; q < 4; ++q) v[q] = i + q < i1 ? ucnt[i + q] : 0u;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) mine += v[q];
+  }
+  uint64_t tot;
+  uint32_t run = (uint32_t)block_exclusive_scan_n<kPlanThreads>(mine, s_scan, &tot);
+  for (uint32_t i = i0; i < i1; i += 4) {
+    uint32_t v[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) v[q] = i + q < i1 ? ucnt[i + q] : 0u;
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+      if (i + q < i1) { upre[i + q] = run; run += v[q]; }
   }
   if (tid == 0) {
     uint64_t nent = 0;
@@ -475,9 +490,9 @@ __global__ void __launch_bounds__(kPlanThreads) ucount_scan_kernel(const __grid_
       const uint32_t* st = starts + (uint64_t)l * (num_w + 1);
       nent += st[num_w] - st[0];
     }
-    ctl->nnz = s_carry;
+    ctl->nnz = tot;
     ctl->nent = nent;
-    if (d_out_nnz) *d_out_nnz = s_carry;
+    if (d_out_nnz) *d_out_nnz = tot;
   }
 }
 
@@ -768,7 +783,7 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
     keep_groups = 1;
   }
   LD_LAUNCH("merge_plan", s, plan_kernel, 1, kPlanThreads, 0, ls.L, starts, M.num_w, G, sparse_max, keep_groups, ctl,
-            items);
+            items, reinterpret_cast<uint32_t*>(w + M.ucnt));
 
   const int grid = (int)(M.num_w < 6u * kNumSMs ? M.num_w : 6u * kNumSMs);   // 6 CTAs/SM (37 KB smem)
   uint32_t* ucnt = reinterpret_cast<uint32_t*>(w + M.ucnt);
