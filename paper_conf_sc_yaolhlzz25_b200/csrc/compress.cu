@@ -1372,17 +1372,57 @@ select_small_kernel(float* __restrict__ r, uint64_t k, Ctl* ctl, const float* __
     }
     __syncthreads();
   };
-  digit(s_h0, 12, 0u, 31, shift(0));               // (the stream pass's histogram is relative to T)
-  const uint32_t d0 = (uint32_t)small_find<bins(0)>(s_h0, need, &above, s_scan);
-  need -= above;
-  digit(s_h1, 10, d0, shift(0), shift(1));
-  const uint32_t d1 = (uint32_t)small_find<bins(1)>(s_h1, need, &above, s_scan);
-  need -= above;
-  const uint32_t p1 = (d0 << 10) | d1;
-  digit(s_h2, 9, p1, shift(1), shift(2));
-  const uint32_t d2 = (uint32_t)small_find<bins(2)>(s_h2, need, &above, s_scan);
-  need -= above;
-  const uint32_t K = (p1 << 9) | d2;
+  // Warm first pass: the stream pass's histogram is fine and relative to T, so the k-th key's bin
+  // b* is found there and ONE pass over the candidates in b* (their low s key bits) gives K*.
+  const uint32_t T = ctl->t_est, FS = ctl->fine_shift;
+  uint32_t K;
+  bool fine = false;
+  if (FS <= 12) {
+    for (int b = tid; b < bins(0); b += kSmallThreads) s_h0[b] = __ldcg(hc + b);
+    __syncthreads();
+    const int bst = small_find<bins(0)>(s_h0, need, &above, s_scan);
+    fine = bst >= 0 && bst < 4095;                 // (uniform) K* below the top (overflow) bin
+    if (fine) {
+      need -= above;
+      __syncthreads();
+      for (int b = tid; b < bins(0); b += kSmallThreads) s_h0[b] = 0;
+      __syncthreads();
+      const uint32_t lowmask = (1u << FS) - 1;
+      for (uint32_t jw = tid & ~31u; jw < cc; jw += kSmallThreads) {   // warp-uniform trip count
+        const uint32_t j = jw + lane;
+        const uint32_t key = j < cc ? mag_key(cand_val[j]) : 0u;
+        const bool take = j < cc && fine_bin(key, T, FS) == (uint32_t)bst;
+        const uint32_t act = __ballot_sync(0xFFFFFFFFu, take);
+        if (take) {
+          const uint32_t bin = (key - T) & lowmask;
+          const uint32_t peers = __match_any_sync(act, bin);
+          if (lane == __ffs(peers) - 1) atomicAdd(&s_h0[bin], (uint32_t)__popc(peers));
+        }
+      }
+      __syncthreads();
+      const uint32_t d = (uint32_t)small_find<bins(0)>(s_h0, need, &above, s_scan);
+      need -= above;
+      K = T + ((uint32_t)bst << FS) + d;
+    } else {
+      need = k;
+      __syncthreads();
+      for (int b = tid; b < bins(0); b += kSmallThreads) s_h0[b] = 0;
+      __syncthreads();
+    }
+  }
+  if (!fine) {                                     // the general 3-digit radix select
+    digit(s_h0, 12, 0u, 31, shift(0));
+    const uint32_t d0 = (uint32_t)small_find<bins(0)>(s_h0, need, &above, s_scan);
+    need -= above;
+    digit(s_h1, 10, d0, shift(0), shift(1));
+    const uint32_t d1 = (uint32_t)small_find<bins(1)>(s_h1, need, &above, s_scan);
+    need -= above;
+    const uint32_t p1 = (d0 << 10) | d1;
+    digit(s_h2, 9, p1, shift(1), shift(2));
+    const uint32_t d2 = (uint32_t)small_find<bins(2)>(s_h2, need, &above, s_scan);
+    need -= above;
+    K = (p1 << 9) | d2;
+  }
   const uint64_t m = need;                         // K*-ties to keep (lowest indices first)
   if (tid == 0) {
     ctl->mode = 0; ctl->kstar = K; ctl->m = m; ctl->small_done = 1;
