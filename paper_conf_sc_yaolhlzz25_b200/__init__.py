@@ -19,7 +19,7 @@ import os
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-SO_PATH = os.path.join(_HERE, "liblowdiff.so")
+SO_PATH = os.environ.get("LOWDIFF_SO") or os.path.join(_HERE, "liblowdiff.so")   # (override: variant experiments)
 
 F32, BF16 = 0, 1
 SUM, STACK = 0, 1

@@ -21,8 +21,8 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
-SO = os.path.join(HERE, "liblowdiff.so")
-BUILD = os.path.join(HERE, "_build")
+SO = os.environ.get("LOWDIFF_SO") or os.path.join(HERE, "liblowdiff.so")
+BUILD = os.environ.get("LOWDIFF_BUILD_DIR") or os.path.join(HERE, "_build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 CFLAGS = ["-O3", "-lineinfo", "-std=c++17", "-fmad=false", "-Xcompiler", "-fPIC",
