@@ -444,12 +444,13 @@ lowdiff_status lowdiff_optimal_config(const lowdiff_config_model* m, double* f_s
  *     "merge_pack", "replay_dense", "replay_sparse", "starts".
  * ------------------------------------------------------------------------------------------- */
 uint64_t       lowdiff_launch_count(void);
-/* After a lowdiff_compress on `stream` with workspace `ws` (syncs the stream): out8 = {first-pass
+/* After a lowdiff_compress on `stream` with workspace `ws` (syncs the stream): out10 = {first-pass
  * threshold key, first-pass candidates found, path (3 = first-pass candidates, fast select; 0 =
  * first-pass candidates, general select; 2 = rescan candidates; 1 = full-array select), k-th key,
- * ties kept, candidate capacity, fine-histogram shift, candidates in the k-th key's fine bin}. */
+ * ties kept, candidate capacity, fine-histogram shift, candidates in the k-th key's fine bin,
+ * rescan threshold key, rescan candidates}. */
 lowdiff_status lowdiff_compress_stats(const void* ws, uint64_t n, uint64_t k, lowdiff_stream_t stream,
-                                      uint64_t* out8);
+                                      uint64_t* out10);
 /* The threshold state of the residual `ws` was last used with (syncs `stream`): out9 =
  * {calls, rescans (path 2), full-array fallbacks (path 1), calls that saw non-finite a, non-finite
  * count of the last call, first-pass candidates of the last call, last k-th key, margin x 2^32,

@@ -713,10 +713,10 @@ def compress_stats(n: int, k: int, device="cuda", stream=None, ws=None) -> dict:
     select, 2 = rescan recovery, 1 = exact full-array select."""
     if ws is None:
         ws = workspace(compress_workspace_size(n, k), device, "compress")
-    out = (C.c_uint64 * 8)()
+    out = (C.c_uint64 * 10)()
     _check(lib().lowdiff_compress_stats(_cuda(ws, "ws"), n, k, _stream(stream), out), "compress_stats")
-    d = dict(zip(("t_est", "candidates", "path", "kstar", "ties_kept", "capacity", "fine_shift", "inbin"),
-                 list(out)))
+    d = dict(zip(("t_est", "candidates", "path", "kstar", "ties_kept", "capacity", "fine_shift", "inbin",
+                  "t2", "candidates2"), list(out)))
     d["fallback"] = int(d["path"] == 1)
     d["rescan"] = int(d["path"] == 2)
     d["first_pass"] = int(d["path"] in (0, 3))

@@ -617,9 +617,9 @@ lowdiff_status lowdiff_compress_counters(const void* ws, lowdiff_stream_t stream
 }
 
 lowdiff_status lowdiff_compress_stats(const void* ws, uint64_t n, uint64_t k, lowdiff_stream_t stream,
-                                      uint64_t* out8) {
-  if (!ws || !out8) return fail(LOWDIFF_EINVAL, "compress_stats: null");
-  return compress_stats(ws, n, k, out8, (cudaStream_t)stream);
+                                      uint64_t* out10) {
+  if (!ws || !out10) return fail(LOWDIFF_EINVAL, "compress_stats: null");
+  return compress_stats(ws, n, k, out10, (cudaStream_t)stream);
 }
 
 lowdiff_status lowdiff_profile_enable(int32_t on) {

@@ -241,7 +241,15 @@ __device__ int find_bin_desc(const uint32_t* h, uint64_t need, uint64_t* above_o
 // micro-chunks first, first + step, ...
 __device__ __forceinline__ void sample_accumulate(const float* r, uint64_t n, uint32_t num_micro, double stride,
                                                   double phase, int exhaustive, uint32_t* sh, uint32_t first,
-                                                  uint32_t step) {
+                                                  uint32_t step, uint32_t* shf = nullptr, uint32_t T = 0,
+                                                  uint32_t t_lo = 0, uint32_t sf = 0) {
+  // shf (optional): keys in [t_lo, T) by their distance below T, bins of 2^sf key units
+  auto fine = [&](uint32_t key) {
+    if (shf && key < T && key >= t_lo) {
+      const uint32_t j = (T - 1 - key) >> sf;      // stored reversed: bin 4095 - j (top = just below T)
+      atomicAdd(&shf[4095u - (j < 4095u ? j : 4095u)], 1u);
+    }
+  };
   const uint64_t n8 = n / 8;
   for (uint32_t m = first; m < num_micro; m += step) {
     uint64_t c8 = exhaustive ? m : (uint64_t)(((double)m + phase) * stride);
@@ -252,9 +260,15 @@ __device__ __forceinline__ void sample_accumulate(const float* r, uint64_t n, ui
       const float4 r1 = __ldcg(reinterpret_cast<const float4*>(r + i + 4));
       const float a[8] = {r0.x, r0.y, r0.z, r0.w, r1.x, r1.y, r1.z, r1.w};
 #pragma unroll
-      for (int e = 0; e < 8; ++e) atomicAdd(&sh[mag_key(a[e]) >> shift(0)], 1u);
+      for (int e = 0; e < 8; ++e) {
+        atomicAdd(&sh[mag_key(a[e]) >> shift(0)], 1u);
+        fine(mag_key(a[e]));
+      }
     } else {
-      for (uint64_t j = i; j < n; ++j) atomicAdd(&sh[mag_key(__ldcg(r + j)) >> shift(0)], 1u);
+      for (uint64_t j = i; j < n; ++j) {
+        atomicAdd(&sh[mag_key(__ldcg(r + j)) >> shift(0)], 1u);
+        fine(mag_key(__ldcg(r + j)));
+      }
     }
   }
 }
@@ -1094,17 +1108,44 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(SelArgs A) {
     } else {
       // too few: a stratified sample of the keys (the first pass's candidates read as their
       // as-if-selected residual: a bias of < k keys, covered by the 2x margin; exhaustive
-      // sampling asks for the k - cc still missing instead)
-      for (int j = threadIdx.x; j < bins(0); j += kThreads) sh[j] = 0;
+      // sampling asks for the k - cc still missing instead). Warm calls (T finite) also histogram
+      // the sampled keys in the eighth below T finely, relative to T: in error-feedback steady
+      // state the keys pile up right below the threshold, and the k-th key usually missed T by a
+      // hair, so T2 is placed where the sample counts max(2 (k - cc), 64 samples' worth) keys in
+      // [T2, T) — the coarse bins alone put T2 percents lower, past the candidate capacity (C5
+      // with a 4-gradient cycle: 3 of 6 rescans overflowed into the full-array select).
+      const bool warm = T < 0x7F800000u;
+      const uint32_t t_lo = warm ? (__float_as_uint(__uint_as_float(T) * 0.875f) & 0x7FFFFFFFu) : 0u;
+      uint32_t sf = 0;
+      while (warm && (4096ull << sf) < (uint64_t)(T - t_lo)) ++sf;
+      uint32_t* shf = reinterpret_cast<uint32_t*>(s_raw + 4 * kTile);   // (the overlay space, free here)
+      for (int j = threadIdx.x; j < bins(0); j += kThreads) { sh[j] = 0; shf[j] = 0; }
       __syncthreads();
       sample_accumulate(A.r, n, A.num_micro, A.stride, A.phase, A.exhaustive, sh,
-                        blockIdx.x * kThreads + threadIdx.x, gridDim.x * kThreads);
+                        blockIdx.x * kThreads + threadIdx.x, gridDim.x * kThreads,
+                        warm ? shf : nullptr, T, t_lo, sf);
       __syncthreads();
-      for (int j = threadIdx.x; j < bins(0); j += kThreads)
+      for (int j = threadIdx.x; j < bins(0); j += kThreads) {
         if (sh[j]) atomicAdd(A.hs + j, sh[j]);
+        if (shf[j]) atomicAdd(A.hl + j, shf[j]);
+      }
       grid.sync();
       uint32_t t2 = threshold_from_sample(A.hs, n, k, k - cc, 2.0, A.num_micro, A.exhaustive, s_scan[0]);
       if (t2 >= T) t2 = __float_as_uint(__uint_as_float(T) * 0.875f) & 0x7FFFFFFFu;
+      if (warm) {
+        // fine placement: bin 4095 - j of hl counts sampled keys in [T - (j+1) 2^sf, T - j 2^sf);
+        // the bin holding the need-th sampled key below T, from the top
+        const uint64_t S = A.exhaustive ? n : (uint64_t)A.num_micro * 8;
+        uint64_t need = (uint64_t)(2.0 * (double)(k - cc) * (double)S / (double)n) + 1;
+        if (need < 64) need = 64;
+        uint64_t above;
+        const int bf = find_bin_desc<bins(0)>(A.hl, need, &above, s_scan[0]);
+        if (bf >= 0) {
+          const uint64_t tf = (uint64_t)T - ((uint64_t)(4096 - bf) << sf);
+          const uint32_t tfine = tf > t_lo ? (uint32_t)tf : t_lo;
+          if (tfine > t2) t2 = tfine;              // the finer (higher) of the two placements
+        }
+      }
       if (threadIdx.x == 0) s_t2 = t2;
     }
     __syncthreads();
@@ -1589,7 +1630,7 @@ void compress_force_threshold(int which, int enable, uint32_t key) {
   (which == 0 ? g_force_t : g_force_t2) = enable ? key : kNoForce;
 }
 
-lowdiff_status compress_stats(const void* ws, uint64_t n, uint64_t k, uint64_t out[8], cudaStream_t s) {
+lowdiff_status compress_stats(const void* ws, uint64_t n, uint64_t k, uint64_t out[10], cudaStream_t s) {
   const Layout L = layout(n, k);
   Ctl c;
   LD_CUDA(cudaMemcpyAsync(&c, static_cast<const uint8_t*>(ws) + L.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s),
@@ -1599,6 +1640,8 @@ lowdiff_status compress_stats(const void* ws, uint64_t n, uint64_t k, uint64_t o
   out[5] = L.cap;
   out[6] = c.fine_shift;
   out[7] = c.inbin_count;
+  out[8] = c.t2;
+  out[9] = c.cand_count2;
   return LOWDIFF_OK;
 }
 

@@ -40,7 +40,7 @@ inline uint64_t align256(uint64_t x) { return (x + 255u) & ~(uint64_t)255u; }
 // ---- compress (compress.cu) ---------------------------------------------------------------
 uint64_t compress_ws_bytes(uint64_t n, uint64_t k);
 void compress_force_threshold(int which /* 0 first pass, 1 rescan */, int enable, uint32_t key);
-lowdiff_status compress_stats(const void* ws, uint64_t n, uint64_t k, uint64_t out[8], cudaStream_t s);
+lowdiff_status compress_stats(const void* ws, uint64_t n, uint64_t k, uint64_t out[10], cudaStream_t s);
 lowdiff_status compress_counters(const void* ws, cudaStream_t s, uint64_t out[9]);
 lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t n, uint64_t k,
                             void* pairs, int vdt, void* ws, cudaStream_t s);

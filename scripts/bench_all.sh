@@ -5,7 +5,7 @@ for C in ${CONFIGS:-1 2 3 4 5}; do
   EXTRA=""
   [ $C = 5 ] && EXTRA="--grad-pool 4"
   [ $C = 4 ] && EXTRA="--grad-pool 8"
-  timeout 900 python bench.py --config $C --steps 10 --warmup 3 --no-e2e --no-cpu-baseline $EXTRA > $OUT/bench_C${C}_$TAG.json 2> $OUT/bench_C${C}_$TAG.err
+  timeout 900 python bench.py --config $C --steps 20 --warmup 5 --no-e2e --no-cpu-baseline $EXTRA > $OUT/bench_C${C}_$TAG.json 2> $OUT/bench_C${C}_$TAG.err
   echo "C$C rc=$?"; tail -2 $OUT/bench_C${C}_$TAG.err
   python -c "
 import json;d=json.load(open('$OUT/bench_C${C}_$TAG.json'))

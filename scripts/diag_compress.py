@@ -38,6 +38,6 @@ for it in range(a.iters):
         print(f"it {it:4d} cand/k {st['candidates'] / cfg.k:7.3f} cap/k {st['capacity'] / cfg.k:6.2f} "
               f"path {st['path']} t_est {f(st['t_est']):.6g} kstar {f(st['kstar']):.6g} "
               f"ratio {f(st['t_est']) / max(f(st['kstar']), 1e-30):.4f} S {st['fine_shift']} inbin {st['inbin']} "
-              f"ties {st['ties_kept']}", flush=True)
+              f"ties {st['ties_kept']} t2 {f(st['t2']):.6g} cand2/k {st['candidates2'] / cfg.k:.3f}", flush=True)
 print(f"fallbacks: {fallbacks} rescans: {rescans} / {a.iters}")
 print(ld.compress_counters(cfg.n, cfg.k))

@@ -13,7 +13,7 @@ bash scripts/bench_all.sh $TAG
 CMD="python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu-baseline"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_$TAG.csv $CMD > /dev/null 2>&1
 echo "ncu launches rc=$?"
-for K in stream_kernel select_kernel sample_kernel merge_kernel dense_kernel; do
+for K in stream_kernel select_kernel merge_kernel dense_kernel starts4_kernel; do
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:$K -s 3 -c 1 -f -o $OUT/prof_${K}_$TAG $CMD > /dev/null 2>&1
   echo "ncu $K rc=$?"
 done
