@@ -48,7 +48,7 @@ _STATE_KEYS = ("x", "m", "v")
 class LowDiffLoop:
     def __init__(self, x: torch.Tensor, opt: dict, lr: float, rho: float, B: int, full_every: int,
                  comm=None, rank: int = 0, world: int = 1, adam_step: int = 0, checkpoint: bool = True,
-                 retain_fulls: int | None = 2, param_group=None):
+                 retain_fulls: int | None = 2, param_group=None, p2p=None):
         assert x.dtype == torch.float32 and x.is_cuda and x.dim() == 1
         assert retain_fulls is None or retain_fulls >= 1
         self.n = x.numel()
@@ -56,6 +56,9 @@ class LowDiffLoop:
         self.k, self.lo, self.hi = self.plan.k, self.plan.lo, self.plan.hi
         self.world, self.comm, self.opt = world, comm, dict(opt)
         self.x_full, self.param_group = x, param_group
+        # world > 1: the Sync is the fused peer-memory one when a lowdiff P2P handle is given
+        # (compress writes straight into this rank's exchange window), else ncclAllGather + coalesce
+        self.p2p = p2p
         self.lr = float(np.float32(lr))
         self.B, self.full_every, self.retain_fulls = B, full_every, retain_fulls
         dev = x.device
@@ -124,6 +127,9 @@ class LowDiffLoop:
         idx, val, nnz = self.slots[slot]
         if self.zero_copy:
             compress(grad, self.r, self.k, pairs=self.pair_slots[slot])
+        elif self.p2p is not None:
+            pairs = compress(grad, self.r, self.k, pairs=self.p2p.slot())
+            self.p2p.allgather_sparse(pairs, self.lo, self.hi, True, out_idx=idx, out_val=val, d_nnz=nnz)
         else:
             pairs = compress(grad, self.r, self.k, pairs=self.pairs)
             allgather_sparse(self.comm, pairs, self.k, "f32", self.lo, self.hi, out_idx=idx, out_val=val,

@@ -164,3 +164,64 @@ def test_p2p_processes_ipc(world, vdt):
     for p in procs:
         p.join(timeout=60)
     assert results == {r: "ok" for r in range(world)}, results
+
+
+def _loop_worker(rank, world, port, q):
+    """One rank of the in-loop driver over the fused peer-memory Sync: per iteration compress into
+    the exchange window, the P2P coalesce of this rank's shard, the live update, and LowDiff's
+    checkpoint side. Checks: the coalesced G~ equals the oracle's coalesce of every rank's pairs
+    (recomputed from the same seeds), and the recovered shard equals the live one bit for bit."""
+    try:
+        import torch.distributed as dist
+        from paper_conf_sc_yaolhlzz25_b200.loop import LowDiffLoop
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        torch.cuda.set_device(0)
+        n, T, B = 200_003, 8, 4
+        k = ld.k_for_density(n, 0.01)
+        h = ld.P2P(world, rank, k, "f32", device="cuda:0")
+        w = torch.zeros(n, device="cuda")
+        opt = {"kind": "adam", "beta1": 0.9, "beta2": 0.999, "eps": 1e-8}
+        loop = LowDiffLoop(w, opt, lr=1e-3, rho=0.01, B=B, full_every=8, world=world, rank=rank,
+                           retain_fulls=None, p2p=h)
+        r_o = [np.zeros(n, np.float32) for _ in range(world)]
+        for t in range(T):
+            gs = [(np.random.default_rng(1000 * t + p).standard_normal(n) * 0.1).astype(np.float32)
+                  for p in range(world)]
+            loop.step(torch.from_numpy(gs[rank]).cuda())
+            pairs = []
+            for p in range(world):
+                oi, ov, r_o[p] = oracle.compress(gs[p], r_o[p], k)
+                pairs.append(oracle.pairs_pack(oi, ov))
+            torch.cuda.synchronize()
+            h.status()
+            idx, val, d_nnz = loop.ring[-1][:3] if loop.ring else loop.slots[(len(loop.slots) - 1)]
+            check(pairs, k, "f32", loop.lo, loop.hi, True, idx, val, d_nnz)
+        live = [loop.state[key].clone() for key in ("x", "m", "v")]
+        rec = loop.recover(T)
+        for a, b in zip((rec["x"], rec["m"], rec["v"]), live):
+            assert torch.equal(a.view(torch.int32), b.view(torch.int32))
+        dist.barrier()
+        h.destroy()
+        dist.destroy_process_group()
+        q.put((rank, "ok"))
+    except Exception:  # pragma: no cover - reported to the parent
+        import traceback
+        q.put((rank, traceback.format_exc()))
+
+
+def test_in_loop_over_p2p_processes():
+    """LowDiffLoop (in-loop LowDiff) with the fused peer-memory Sync at world 2:
+    two processes sharing the GPU through CUDA IPC (round 1's P2P loop stalled and was not shipped)."""
+    import torch.multiprocessing as mp
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_loop_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    results = dict(q.get(timeout=600) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+    assert results == {r: "ok" for r in range(world)}, results
