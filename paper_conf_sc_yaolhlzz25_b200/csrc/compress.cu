@@ -850,7 +850,14 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
   const uint64_t k = A.k;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t lowmask = (1u << S) - 1;
-  const uint32_t CH = A.chunk_tiles, num_tiles = A.num_tiles;
+  const uint32_t num_tiles = A.num_tiles;
+  // chunking of the tile counts: tiles holding >= 32 candidates (C2, C4) go through long runs with a
+  // warp-wide prefix over chunks of 32q tiles; sparser tiles take the finest chunks kMaxChunks allows
+  // so each lane can sum its own tile's prefix (measured: C3 select 45.8 -> 37.6 us; the finer
+  // chunks cost the dense-tile configurations their longer chunk-offset prologue)
+  const bool dense_tiles = cc / (num_tiles ? num_tiles : 1) >= 32;
+  const uint32_t CH = dense_tiles || num_tiles == 0 ? A.chunk_tiles : (num_tiles + kMaxChunks - 1) / kMaxChunks;
+  const uint32_t nch = (num_tiles + CH - 1) / CH;
   constexpr uint64_t kGt = 1ull << 32;             // packed count: (> K*) << 32 | (== K*)
   float* r = A.r;
   const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
@@ -948,7 +955,6 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
   // ---- phase 3: chunk offsets (every CTA), then the ordered emission ----
   uint64_t* s_coff = reinterpret_cast<uint64_t*>(s_raw);          // <= 4096 chunks
   {
-    const uint32_t nch = A.num_chunks;
     const uint32_t per = (nch + kThreads - 1) / kThreads;         // <= 16
     uint64_t v[16], gsum = 0, esum = 0;
 #pragma unroll
@@ -985,7 +991,8 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
   const uint32_t lt = (1u << lane) - 1;
   // (measured: one word per run when tiles hold < 32 candidates, C2/C3; one contiguous range per
   // warp above, C4)
-  const uint64_t W = (cc / (num_tiles ? num_tiles : 1)) >= 32 ? ((cc + nwarps * 32 - 1) / (nwarps * 32)) : 1;
+  const uint64_t W = dense_tiles ? ((cc + nwarps * 32 - 1) / (nwarps * 32)) : 1;
+  const bool lane_prefix = !dense_tiles && CH <= 16;   // (uniform)
   for (uint64_t run0 = wid * 32 * W; run0 < cc; run0 += nwarps * 32 * W) {   // warp-uniform
   const uint64_t p_end = run0 + 32 * W < cc ? run0 + 32 * W : cc;
   uint32_t cur_t = 0xFFFFFFFFu;                    // the tile continuing from the previous word
@@ -1014,8 +1021,34 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
     const float a = n_a;
     if (base + 32 < p_end) load_word(base + 32);
     const uint32_t t = in ? idx / kTile : 0xFFFFFFFFu;
-    uint32_t pend = __ballot_sync(0xFFFFFFFFu, in);
     uint64_t before = 0;
+    if (lane_prefix) {
+      // one word per run and short chunks: each lane sums its own tile's prefix (chunk offset +
+      // < CH tile counts, independent loads; lanes of one tile repeat it) — no warp-wide loop over
+      // the word's distinct tiles. Only the word's first tile can have begun in an earlier word.
+      const uint32_t peers = __match_any_sync(0xFFFFFFFFu, t);
+      const uint32_t first = (uint32_t)__ffs(peers) - 1;
+      uint64_t b0 = 0;
+      if (in) {
+        const uint32_t cb = t / CH * CH;
+        b0 = s_coff[t / CH];
+        for (uint32_t j = cb; j < t; ++j) b0 += __ldcg(A.tk + j);
+      }
+      const uint32_t sx0 = __shfl_sync(0xFFFFFFFFu, in ? A.tinfo1[t].x : 0u, 0);
+      if (sx0 < base) {                            // warp-uniform (lane 0 is always in)
+        uint64_t c = 0;
+        for (uint64_t w = (sx0 >> 5) + lane; w < (base >> 5); w += 32) {
+          uint32_t g1 = __ldcg(A.gbits + w), e1 = __ldcg(A.ebits + w);
+          if (w == (sx0 >> 5)) { g1 &= ~((1u << (sx0 & 31)) - 1); e1 &= ~((1u << (sx0 & 31)) - 1); }
+          c += ((uint64_t)__popc(g1) << 32) | __popc(e1);
+        }
+        c = warp_sum64(c);
+        if (first == 0) b0 += c;                    // lane 0's tile: its lanes start at lane 0
+      }
+      const uint32_t msk = lt & ~((1u << first) - 1);
+      before = b0 + (((uint64_t)__popc(gw & msk)) << 32) + __popc(ew & msk);
+    }
+    uint32_t pend = lane_prefix ? 0u : __ballot_sync(0xFFFFFFFFu, in);
     uint32_t last_t = 0xFFFFFFFFu;
     uint64_t last_before = 0;
     while (pend) {                                 // warp-uniform: each distinct tile of this word
@@ -1047,8 +1080,10 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
       last_t = tt;
       last_before = b0 + (((uint64_t)__popc(gw & same)) << 32) + __popc(ew & same);
     }
-    cur_t = last_t;                                // the word's last tile may continue
-    cur_before = last_before;
+    if (!lane_prefix) {
+      cur_t = last_t;                              // the word's last tile may continue
+      cur_before = last_before;
+    }
     const bool isg = in && ((gw >> lane) & 1u), ise = in && ((ew >> lane) & 1u);
     const uint64_t gtb = before >> 32, eqb = before & 0xFFFFFFFFull;
     if (isg || (ise && eqb < m)) {
@@ -1755,7 +1790,7 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   A.inbin = reinterpret_cast<uint64_t*>(w + L.inbin);
   {
     const uint32_t q = (L.num_tiles + 32u * kMaxChunks - 1) / (32u * kMaxChunks);
-    A.chunk_tiles = 32u * (q ? q : 1u);
+    A.chunk_tiles = 32u * (q ? q : 1u);            // dense tiles; fast_select picks finer for sparse
     A.num_chunks = (L.num_tiles + A.chunk_tiles - 1) / A.chunk_tiles;
   }
   A.boff = reinterpret_cast<uint64_t*>(w + L.boff);
