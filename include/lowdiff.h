@@ -328,6 +328,9 @@ typedef struct {
 } lowdiff_record_view;
 
 lowdiff_status lowdiff_record_parse(const void* h_bytes, uint64_t len, lowdiff_record_header* out);
+/* Workspace: 256 B error word + a starts table (4 B per record per 256-parameter warp tile of
+ * [lo, hi)) + 2 B per entry of every STACK record (its (it, position) repacked for the dense kernel); the
+ * size query reads each record's host header (recs[i].h_head) for mode and entry count. */
 lowdiff_status lowdiff_replay_workspace_size(const lowdiff_state* st, const lowdiff_record_view* recs,
                                              uint32_t nrec, uint64_t* bytes);
 lowdiff_status lowdiff_replay(lowdiff_state* st, const lowdiff_opt* opt,

@@ -475,8 +475,17 @@ static lowdiff_status check_state(const lowdiff_state* st, const lowdiff_opt* o)
 lowdiff_status lowdiff_replay_workspace_size(const lowdiff_state* st, const lowdiff_record_view* recs, uint32_t nrec,
                                              uint64_t* bytes) {
   if (!st || !bytes || st->lo >= st->hi) return fail(LOWDIFF_EINVAL, "replay_workspace_size");
-  (void)recs;
-  *bytes = replay_ws_bytes(st->hi - st->lo, nullptr, nrec) + 256;
+  if (nrec && !recs) return fail(LOWDIFF_EINVAL, "replay_workspace_size: null records");
+  std::vector<RecInfo> R(nrec);                    // only mode and nent size the workspace
+  for (uint32_t q = 0; q < nrec; ++q) {
+    lowdiff_record_header h;
+    if (!recs[q].h_head) return fail(LOWDIFF_EINVAL, "replay_workspace_size: record %u has no host header", q);
+    const lowdiff_status s = lowdiff_record_parse(recs[q].h_head, recs[q].h_head_len, &h);
+    if (s) return s;
+    R[q].mode = h.mode;
+    R[q].nent = h.nent;
+  }
+  *bytes = replay_ws_bytes(st->hi - st->lo, R.data(), nrec) + 256;
   return LOWDIFF_OK;
 }
 

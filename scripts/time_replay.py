@@ -49,8 +49,8 @@ del sig, r, ws, grads
 ck = full_checkpoint(cfg, 0, n, dev)
 xb = torch.empty(n, dtype=torch.bfloat16, device=dev) if cfg.gdt == "bf16" else None
 st = {"x0": ck["x"], "m0": ck["m"], "v0": ck["v"], "x": torch.empty_like(ck["x"]), "m": torch.empty_like(ck["m"]),
-      "v": torch.empty_like(ck["v"]), "x_bf16": xb, "n": n, "lo": 0, "hi": n}
-opt = {"kind": "adam", "beta1": 0.9, "beta2": 0.999, "eps": 1e-8}
+      "v": torch.empty_like(ck["v"]) if ck["v"] is not None else None, "x_bf16": xb, "n": n, "lo": 0, "hi": n}
+opt = {"kind": cfg.opt, **{k2: v2 for k2, v2 in cfg.hyper.items() if k2 != "lr"}}
 clocks, stop = [], [False]
 
 
@@ -66,7 +66,7 @@ def sample():
 def run(reps):
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
     for i in range(reps):
-        st.update(t=0, adam_step=ck["adam_step"], momentum_initialized=0)
+        st.update(t=0, adam_step=ck["adam_step"], momentum_initialized=ck["momentum_initialized"])
         ev[i][0].record()
         ld.replay(st, opt, recs, check=False)
         ev[i][1].record()
