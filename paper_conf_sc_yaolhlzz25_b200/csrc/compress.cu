@@ -843,6 +843,35 @@ __device__ __forceinline__ uint64_t warp_sum64(uint64_t v) {
   return v;
 }
 
+#ifdef LOWDIFF_SEL_TIMING
+// experiment instrumentation (not in the product build): per-CTA %globaltimer stamps at the phase
+// boundaries of the fast select, printed by sel_timing_print for one chosen call
+__device__ uint64_t g_seltime[8][1024];
+__device__ __forceinline__ void sel_stamp(int i) {
+  if (threadIdx.x == 0 && blockIdx.x < 1024) {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    g_seltime[i][blockIdx.x] = t;
+  }
+}
+__global__ void sel_timing_print(const State* st, uint32_t grid, uint64_t when) {
+  if (st->calls != when) return;
+  uint64_t t0 = ~0ull;
+  for (uint32_t b = 0; b < grid; ++b) t0 = min(t0, g_seltime[0][b]);
+  for (int i = 0; i < 8; ++i) {
+    uint64_t lo = ~0ull, hi = 0, sum = 0;
+    for (uint32_t b = 0; b < grid; ++b) {
+      const uint64_t t = g_seltime[i][b] - t0;
+      lo = min(lo, t); hi = max(hi, t); sum += t;
+    }
+    printf("sel stamp %d: min %.2f us  mean %.2f us  max %.2f us\n", i, lo * 1e-3, sum * 1e-3 / grid, hi * 1e-3);
+  }
+}
+#define SEL_STAMP(i) sel_stamp(i)
+#else
+#define SEL_STAMP(i)
+#endif
+
 template <bool VBF16>
 __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t bst, uint64_t above,
                             uint32_t cc, uint8_t* s_raw, uint64_t* s_scan, cg::grid_group& grid) {
@@ -863,6 +892,7 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
   const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
   const uint64_t wid = ((uint64_t)blockIdx.x * kThreads + threadIdx.x) >> 5;
   // ---- phase 1: classify (4 words per warp in flight) ----
+  SEL_STAMP(1);
   constexpr int U1 = 4;
   for (uint64_t base0 = wid * 32; base0 < cc; base0 += U1 * nwarps * 32) {   // warp-uniform
   float av[U1];
@@ -907,7 +937,9 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
     }
   }
   }
+  SEL_STAMP(2);
   grid.sync();
+  SEL_STAMP(3);
   // ---- phase 2: K*, m; resolve this CTA's slice of the undecided ----
   __shared__ uint32_t s_K;
   __shared__ uint64_t s_m;
@@ -951,7 +983,9 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
     ctl->mode = 3; ctl->kstar = K; ctl->m = m;
     state_update(A.st, A.sk, k, A.cap, cc, 3, K, ctl->nonfinite);
   }
+  SEL_STAMP(4);
   grid.sync();
+  SEL_STAMP(5);
   // ---- phase 3: chunk offsets (every CTA), then the ordered emission ----
   uint64_t* s_coff = reinterpret_cast<uint64_t*>(s_raw);          // <= 4096 chunks
   {
@@ -974,6 +1008,7 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
     }
   }
   __syncthreads();
+  SEL_STAMP(6);
   uint8_t* pairs = A.pairs;
   uint32_t* out_idx = reinterpret_cast<uint32_t*>(pairs);
   uint8_t* out_val = pairs + pad16(4 * k);
@@ -1106,6 +1141,7 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(SelArgs A) {
   uint32_t* sh = reinterpret_cast<uint32_t*>(s_raw);
   Ctl* ctl = A.ctl;
   if (ctl->small_done) return;                     // the one-CTA select did this call (uniform)
+  SEL_STAMP(0);
   const uint64_t n = A.n, k = A.k;
   const uint32_t cap = A.cap, num_tiles = A.num_tiles;
   const uint32_t cc = ctl->cand_count;
@@ -1123,6 +1159,7 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(SelArgs A) {
     const uint32_t inb = bst >= 0 ? __ldcg(A.hc + bst) : ~0u;
     if (A.fast && bst >= 0 && bst < 4095 && FS <= 12 && inb <= cap) {
       fast_select<VBF16>(A, T, FS, (uint32_t)bst, above, cc, s_raw, s_scan[0], grid);
+      SEL_STAMP(7);
       return;
     }
   }
@@ -1823,6 +1860,13 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   void* args[] = {(void*)&A};
   LD_CUDA(cudaLaunchCooperativeKernel(select_fn(vbf), sel_grid, kThreads, args, 0, s), "select launch");
   note_launch();
+#ifdef LOWDIFF_SEL_TIMING
+  {
+    static uint64_t when = 0;
+    if (!when) { const char* e = getenv("LOWDIFF_SEL_TIMING_CALL"); when = e ? strtoull(e, nullptr, 10) : 410; }
+    sel_timing_print<<<1, 1, 0, s>>>(st, (uint32_t)sel_grid, when);
+  }
+#endif
   return cuda_status(cudaGetLastError(), "compress launch");
 }
 
