@@ -893,7 +893,15 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
   const uint64_t wid = ((uint64_t)blockIdx.x * kThreads + threadIdx.x) >> 5;
   // ---- phase 1: classify (4 words per warp in flight) ----
   SEL_STAMP(1);
-  constexpr int U1 = 4;
+  constexpr uint32_t kStage = 2 * 4 * kTile / 8;   // undecided entries staged per CTA (s_raw)
+  uint64_t* s_stage = reinterpret_cast<uint64_t*>(s_raw);
+  __shared__ uint32_t s_ucnt;
+  if (threadIdx.x == 0) s_ucnt = 0;
+  __syncthreads();
+#ifndef LOWDIFF_SEL_U1
+#define LOWDIFF_SEL_U1 4
+#endif
+  constexpr int U1 = LOWDIFF_SEL_U1;
   for (uint64_t base0 = wid * 32; base0 < cc; base0 += U1 * nwarps * 32) {   // warp-uniform
   float av[U1];
   uint32_t iv[U1];
@@ -927,15 +935,33 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
     }
     const uint32_t ub = __ballot_sync(0xFFFFFFFFu, und);
     if (ub) {
+      // staged in shared memory and appended to the global list once per CTA (one global counter
+      // for every undecided word serialised phase 1 at C4); the global counter only on overflow
       uint32_t slot0 = 0;
-      if (lane == __ffs(ub) - 1) slot0 = atomicAdd(&ctl->inbin_count, (uint32_t)__popc(ub));
+      if (lane == __ffs(ub) - 1) slot0 = atomicAdd(&s_ucnt, (uint32_t)__popc(ub));
       slot0 = __shfl_sync(0xFFFFFFFFu, slot0, __ffs(ub) - 1);
+      const bool staged = slot0 + __popc(ub) <= kStage;   // (warp-uniform)
+      if (!staged) {
+        if (lane == __ffs(ub) - 1) slot0 = atomicAdd(&ctl->inbin_count, (uint32_t)__popc(ub));
+        slot0 = __shfl_sync(0xFFFFFFFFu, slot0, __ffs(ub) - 1);
+      }
       if (und) {
-        A.inbin[slot0 + __popc(ub & ((1u << lane) - 1))] = ((uint64_t)p << 32) | __float_as_uint(a);
+        const uint64_t ent = ((uint64_t)p << 32) | __float_as_uint(a);
+        const uint32_t sl = slot0 + __popc(ub & ((1u << lane) - 1));
+        if (staged) s_stage[sl] = ent;
+        else A.inbin[sl] = ent;
         atomicAdd(&A.hl[(key - T) & lowmask], 1u);
       }
     }
   }
+  }
+  __syncthreads();
+  {
+    const uint32_t ns = min(s_ucnt, kStage);
+    __shared__ uint32_t s_g0;
+    if (threadIdx.x == 0 && ns) s_g0 = atomicAdd(&ctl->inbin_count, ns);
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i < ns; i += kThreads) A.inbin[s_g0 + i] = s_stage[i];
   }
   SEL_STAMP(2);
   grid.sync();
@@ -990,11 +1016,15 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
   uint64_t* s_coff = reinterpret_cast<uint64_t*>(s_raw);          // <= 4096 chunks
   {
     const uint32_t per = (nch + kThreads - 1) / kThreads;         // <= 16
+    // coalesced into shared memory first (every CTA reads the same lines: thread-contiguous global
+    // reads cost 4x the L2 sector requests), then each thread scans its contiguous run
+    for (uint32_t c = threadIdx.x; c < nch; c += kThreads) s_coff[c] = __ldcg(A.ctot + c);
+    __syncthreads();
     uint64_t v[16], gsum = 0, esum = 0;
 #pragma unroll
     for (int q = 0; q < 16; ++q) {
       const uint32_t c = threadIdx.x * per + q;
-      v[q] = (q < (int)per && c < nch) ? __ldcg(A.ctot + c) : 0ull;
+      v[q] = (q < (int)per && c < nch) ? s_coff[c] : 0ull;
       gsum += v[q] >> 32;
       esum += v[q] & 0xFFFFFFFFull;
     }
