@@ -201,17 +201,28 @@ __device__ void state_update(State* st, const StateKey& sk, uint64_t k, uint32_t
 // ---- histogram "find": the bin holding the need-th largest key (1-based) --------------------
 // h: global histogram (nb bins, nb % 256 == 0). Walks bins from the top. Returns the bin
 // (or -1 if the total is below `need`) and, via *above, the count in strictly higher bins.
+// stage (optional): NB words of shared memory; the histogram is then read coalesced into it first
+// (every CTA of a grid reads the same lines: thread-contiguous global reads cost 4x the L2 requests)
 template <int NB>
-__device__ int find_bin_desc(const uint32_t* h, uint64_t need, uint64_t* above_out, uint64_t* smem_scan) {
+__device__ int find_bin_desc(const uint32_t* h, uint64_t need, uint64_t* above_out, uint64_t* smem_scan,
+                             uint32_t* stage = nullptr) {
   __shared__ int s_bin;
   __shared__ uint64_t s_above;
   constexpr int PER = NB / kThreads;               // 16, 4 or 2 bins per thread, loaded as vectors
   const int lo = NB - (threadIdx.x + 1) * PER;     // this thread's bins: [lo, lo + PER)
   uint32_t c[PER];
+  if (stage) {
+    for (int j = threadIdx.x; j < NB / 4; j += kThreads)
+      reinterpret_cast<uint4*>(stage)[j] = __ldcg(reinterpret_cast<const uint4*>(h) + j);
+    __syncthreads();
 #pragma unroll
-  for (int q = 0; q < PER; q += 2) {
-    const uint2 u = __ldcg(reinterpret_cast<const uint2*>(h + lo + q));
-    c[q] = u.x; c[q + 1] = u.y;
+    for (int q = 0; q < PER; ++q) c[q] = stage[lo + q];
+  } else {
+#pragma unroll
+    for (int q = 0; q < PER; q += 2) {
+      const uint2 u = __ldcg(reinterpret_cast<const uint2*>(h + lo + q));
+      c[q] = u.x; c[q + 1] = u.y;
+    }
   }
   uint64_t sum = 0;
 #pragma unroll
@@ -975,13 +986,16 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
     const uint32_t per = NB > kThreads ? NB / kThreads : 1;
     const bool act = threadIdx.x * per < NB;
     const uint32_t lo = act ? NB - (threadIdx.x + 1) * per : 0;
+    uint32_t* s_hl = reinterpret_cast<uint32_t*>(s_raw);  // coalesced copy (every CTA reads it)
+    for (uint32_t j = threadIdx.x; j < NB; j += kThreads) s_hl[j] = __ldcg(A.hl + j);
+    __syncthreads();
     uint64_t sum = 0;
-    for (uint32_t q = 0; q < per && act; ++q) sum += __ldcg(A.hl + lo + q);
+    for (uint32_t q = 0; q < per && act; ++q) sum += s_hl[lo + q];
     uint64_t tot;
     uint64_t ab = block_exclusive_scan(sum, s_scan, &tot);
     if (act && ab < need && ab + sum >= need) {
       for (int q = (int)per - 1; q >= 0; --q) {
-        const uint32_t c = __ldcg(A.hl + lo + q);
+        const uint32_t c = s_hl[lo + q];
         if (ab + c >= need) { s_K = T + (bst << S) + lo + q; s_m = need - ab; break; }
         ab += c;
       }
@@ -1185,7 +1199,7 @@ __global__ void __launch_bounds__(kThreads, 4) select_kernel(SelArgs A) {
   uint32_t mode = 0;
   if (cc >= k && cc <= cap) {
     uint64_t above;
-    const int bst = find_bin_desc<bins(0)>(A.hc, k, &above, s_scan[0]);
+    const int bst = find_bin_desc<bins(0)>(A.hc, k, &above, s_scan[0], sh);
     const uint32_t inb = bst >= 0 ? __ldcg(A.hc + bst) : ~0u;
     if (A.fast && bst >= 0 && bst < 4095 && FS <= 12 && inb <= cap) {
       fast_select<VBF16>(A, T, FS, (uint32_t)bst, above, cc, s_raw, s_scan[0], grid);
