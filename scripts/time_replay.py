@@ -20,6 +20,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", type=int, default=3)
 ap.add_argument("--reps", type=int, default=20)
 ap.add_argument("--ef-warmup", type=int, default=0, help="EF iterations (gradient cycle of B) before the chain")
+ap.add_argument("--grad-pool", type=int, default=0, help="distinct gradients cycled (default B; C5 needs <= 4)")
 a = ap.parse_args()
 cfg = CONFIGS[a.config]
 dev = torch.device("cuda", 0)
@@ -30,14 +31,15 @@ ws = torch.zeros(ld.compress_workspace_size(n, k), dtype=torch.uint8, device=dev
 slots = [torch.empty(ld.pairs_bytes(k, cfg.vdt), dtype=torch.uint8, device=dev) for _ in range(B)]
 d_k = torch.full((1,), k, dtype=torch.int64, device=dev)
 lr = float(np.float32(cfg.hyper["lr"]))
-grads = [gradient(cfg, 0, t, dev, sigmas=sig) for t in range(B)]
+G = a.grad_pool or B
+grads = [gradient(cfg, 0, t, dev, sigmas=sig) for t in range(G)]
 for t in range(a.ef_warmup):                     # error-feedback steady state, as in the bench
-    ld.compress(grads[t % B], r, k, vdt=cfg.vdt, pairs=slots[0], ws=ws)
+    ld.compress(grads[t % G], r, k, vdt=cfg.vdt, pairs=slots[0], ws=ws)
 recs = []
 for b in range(K // B):
     ring = []
     for j in range(B):
-        ld.compress(grads[j], r, k, vdt=cfg.vdt, pairs=slots[j], ws=ws)
+        ld.compress(grads[j % G], r, k, vdt=cfg.vdt, pairs=slots[j], ws=ws)
         ring.append(ld.pairs_views(slots[j], k, cfg.vdt) + (d_k, k, lr))
     rec, d_bytes = ld.batch_merge(ring, "stack", n, 0, n, b * B, 1)
     nb = ld.record_bytes(d_bytes, rec.numel())
