@@ -895,7 +895,9 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
   // warp-wide prefix over chunks of 32q tiles; sparser tiles take the finest chunks kMaxChunks allows
   // so each lane can sum its own tile's prefix (measured: C3 select 45.8 -> 37.6 us; the finer
   // chunks cost the dense-tile configurations their longer chunk-offset prologue)
-  const bool dense_tiles = cc / (num_tiles ? num_tiles : 1) >= 32;
+  // (tiles of >= 32 candidates take the per-lane prefix too while the fine chunks stay <= 16 tiles:
+  // C2 compress 81 -> 75 us per call; only C4/C5-sized tile counts keep the long warp runs)
+  const bool dense_tiles = cc / (num_tiles ? num_tiles : 1) >= 32 && (num_tiles + kMaxChunks - 1) / kMaxChunks > 16;
   const uint32_t CH = dense_tiles || num_tiles == 0 ? A.chunk_tiles : (num_tiles + kMaxChunks - 1) / kMaxChunks;
   const uint32_t nch = (num_tiles + CH - 1) / CH;
   constexpr uint64_t kGt = 1ull << 32;             // packed count: (> K*) << 32 | (== K*)
