@@ -1840,8 +1840,10 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
 
   const int sel_max = select_max_per_sm();
   // CTAs per SM: more hide the latency of the emission loop at large k, fewer make the grid
-  // syncs and histogram flushes cheaper at small k (measured, profiles/README.md).
-  int want = k >= (1u << 18) ? 4 : 2;
+  // syncs and histogram flushes cheaper at small k (measured, profiles/README.md; round 2 with the
+  // fast select: 3 per SM for 2^14 <= k < 2^18, C2 74.8 -> 73.1 us, C3 289 -> 287.1 us per call;
+  // C1's k = 2697 keeps 2: 19.1 vs 20.5 us)
+  int want = k >= (1u << 18) ? 4 : (k >= (1u << 14) ? 3 : 2);
   if (const char* e = getenv("LOWDIFF_SELECT_PER_SM")) want = atoi(e);
   if (want < 1) want = 1;
   if (want > sel_max) want = sel_max;
