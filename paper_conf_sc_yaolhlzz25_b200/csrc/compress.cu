@@ -1113,7 +1113,13 @@ __device__ void fast_select(const SelArgs& A, uint32_t T, uint32_t S, uint32_t b
       if (in) {
         const uint32_t cb = t / CH * CH;
         b0 = s_coff[t / CH];
-        for (uint32_t j = cb; j < t; ++j) b0 += __ldcg(A.tk + j);
+        // the < CH <= 16 tile counts before t: predicated, unrolled, so the loads go out together
+        // (a rolled loop serialised them: one round trip per tile)
+        uint64_t tv[15];
+#pragma unroll
+        for (int q = 0; q < 15; ++q) tv[q] = cb + q < t ? __ldcg(A.tk + cb + q) : 0ull;
+#pragma unroll
+        for (int q = 0; q < 15; ++q) b0 += tv[q];
       }
       const uint32_t sx0 = __shfl_sync(0xFFFFFFFFu, in ? A.tinfo1[t].x : 0u, 0);
       if (sx0 < base) {                            // warp-uniform (lane 0 is always in)
