@@ -1791,14 +1791,23 @@ lowdiff_status compress_run(const void* grad, int gdt, float* residual, uint64_t
   Ctl* ctl = reinterpret_cast<Ctl*>(w + L.ctl);
   State* st = reinterpret_cast<State*>(w + L.state);
   LD_CUDA(cudaMemsetAsync(w + L.ctl, 0, L.zero_end - L.ctl, s), "memset compress workspace");
-  static float band_lo = 0.f, band_hi = 0.f;
-  if (band_lo == 0.f) {                            // LOWDIFF_CAND_BAND="lo,hi" (experiments)
-    band_lo = 1.05f; band_hi = 1.5f;              // measured: scripts/band_sweep.sh (profiles/r02/band.txt)
+  // the margin controller's band of first-pass candidates / k (measured: scripts/band_sweep.sh,
+  // profiles/r02/band.txt): 1.05-1.5 k; 1.02-1.2 k for large, dense selections (k >= 2^20 and
+  // k >= n/200) — each rejected candidate costs a scattered residual store, ~0.8 M per call at C4
+  // (C4 659 -> 643 us per call). Sparser selections lose to extra rescans with the tight band (C5:
+  // 49 rescans in 1,200 error-feedback calls instead of 1-4; C2, C3 slower).
+  // LOWDIFF_CAND_BAND="lo,hi" overrides (experiments).
+  static float env_lo = -1.f, env_hi = -1.f;
+  if (env_lo < 0.f) {
+    env_lo = env_hi = 0.f;
     if (const char* e = getenv("LOWDIFF_CAND_BAND")) {
       float a = 0.f, b = 0.f;
-      if (sscanf(e, "%f,%f", &a, &b) == 2 && a >= 1.0f && b > a) { band_lo = a; band_hi = b; }
+      if (sscanf(e, "%f,%f", &a, &b) == 2 && a >= 1.0f && b > a) { env_lo = a; env_hi = b; }
     }
   }
+  const bool big_k = k >= (1ull << 20) && 200 * k >= n;
+  const float band_lo = env_lo > 0.f ? env_lo : (big_k ? 1.02f : 1.05f);
+  const float band_hi = env_lo > 0.f ? env_hi : (big_k ? 1.2f : 1.5f);
   const StateKey sk{n, k, (uint64_t)(uintptr_t)residual, (uint64_t)(gdt | (vdt << 8)), band_lo, band_hi};
 
   // recovery sample size: >= 512 expected keys above the k-th (S >= 512 n / k: the 2x target is
