@@ -53,7 +53,8 @@ class RecordHeader(C.Structure):
 class Opt(C.Structure):
     _fields_ = [("kind", C.c_int32), ("momentum", C.c_double), ("dampening", C.c_double),
                 ("weight_decay", C.c_double), ("beta1", C.c_double), ("beta2", C.c_double),
-                ("eps", C.c_double), ("nesterov", C.c_int32), ("allow_accumulated_sum", C.c_int32)]
+                ("eps", C.c_double), ("nesterov", C.c_int32), ("allow_accumulated_sum", C.c_int32),
+                ("approx_math", C.c_int32)]
 
 
 class State(C.Structure):
@@ -578,7 +579,8 @@ def _replay_args(state: dict, opt: dict, records):
     import numpy as np
     o = Opt(_KIND[opt["kind"]], opt.get("momentum", 0.0), opt.get("dampening", 0.0),
             opt.get("weight_decay", 0.0), opt.get("beta1", 0.9), opt.get("beta2", 0.999),
-            opt.get("eps", 1e-8), int(opt.get("nesterov", 0)), int(opt.get("allow_accumulated_sum", 0)))
+            opt.get("eps", 1e-8), int(opt.get("nesterov", 0)), int(opt.get("allow_accumulated_sum", 0)),
+            int(opt.get("approx_math", 0)))
     ptr = lambda key: _cuda(state[key], key) if state.get(key) is not None else None
     st = State(ptr("x"), ptr("m"), ptr("v"), ptr("x_bf16"), state["n"], state["lo"], state["hi"],
                state["t"], state["adam_step"], state["momentum_initialized"],

@@ -21,6 +21,7 @@ ap.add_argument("--config", type=int, default=3)
 ap.add_argument("--reps", type=int, default=20)
 ap.add_argument("--ef-warmup", type=int, default=0, help="EF iterations (gradient cycle of B) before the chain")
 ap.add_argument("--grad-pool", type=int, default=0, help="distinct gradients cycled (default B; C5 needs <= 4)")
+ap.add_argument("--approx", type=int, default=0, help="lowdiff_opt.approx_math (Adam: MUFU sqrt/rcp)")
 a = ap.parse_args()
 cfg = CONFIGS[a.config]
 dev = torch.device("cuda", 0)
@@ -52,7 +53,7 @@ ck = full_checkpoint(cfg, 0, n, dev)
 xb = torch.empty(n, dtype=torch.bfloat16, device=dev) if cfg.gdt == "bf16" else None
 st = {"x0": ck["x"], "m0": ck["m"], "v0": ck["v"], "x": torch.empty_like(ck["x"]), "m": torch.empty_like(ck["m"]),
       "v": torch.empty_like(ck["v"]) if ck["v"] is not None else None, "x_bf16": xb, "n": n, "lo": 0, "hi": n}
-opt = {"kind": cfg.opt, **{k2: v2 for k2, v2 in cfg.hyper.items() if k2 != "lr"}}
+opt = {"kind": cfg.opt, **{k2: v2 for k2, v2 in cfg.hyper.items() if k2 != "lr"}, "approx_math": a.approx}
 clocks, stop = [], [False]
 
 
@@ -82,6 +83,6 @@ th.start()
 ms = run(a.reps)
 stop[0] = True
 th.join()
-print(json.dumps({"config": cfg.name, "ef_warmup": a.ef_warmup, "replay_ms_median": float(np.median(ms)), "replay_ms_min": min(ms),
+print(json.dumps({"config": cfg.name, "ef_warmup": a.ef_warmup, "approx": a.approx, "replay_ms_median": float(np.median(ms)), "replay_ms_min": min(ms),
                   "sm_mhz_median": float(np.median(clocks)) if clocks else None,
                   "sm_mhz_min": min(clocks) if clocks else None, "clock_samples": len(clocks)}))
