@@ -49,14 +49,13 @@ struct __align__(256) MCtl {
 // ENTRY offset (known from the starts table alone, so items need no ordering between them); a
 // scan over the items' unique counts and a compaction then place them densely.
 struct MLayout {
-  uint64_t ctl, ebnd, zero_end, starts, items, ucnt, epre, upre, sidx, sval, widx, wval, wit, went, total;
+  uint64_t ctl, ebnd, zero_end, starts, items, ucnt, epre, upre, sidx, sval, wit, went, total;
   uint32_t num_w;
 };
 
 MLayout mlayout(int L, uint64_t max_entries, uint64_t lo, uint64_t hi, bool record) {
   MLayout M;
   M.num_w = (uint32_t)((hi - lo + kW - 1) / kW);
-  const uint64_t cap_u = max_entries < hi - lo ? max_entries : hi - lo;
   uint64_t o = 0;
   M.ctl = o;    o += align256(sizeof(MCtl));
   M.zero_end = o;
@@ -68,10 +67,9 @@ MLayout mlayout(int L, uint64_t max_entries, uint64_t lo, uint64_t hi, bool reco
   M.upre = o;   o += align256(4ull * M.num_w);   // unique offset per item (scan)
   M.sidx = o;   o += align256(4 * max_entries);  // staged heads: idx
   M.sval = o;   o += align256(4 * max_entries);  // staged heads: value (SUM/coalesce) or off (STACK)
-  M.widx = M.wval = M.wit = M.went = 0;
-  if (record) {
-    M.widx = o; o += align256(4 * cap_u);
-    M.wval = o; o += align256(4 * cap_u);         // SUM values, or STACK off[] (u32)
+  M.wit = M.went = 0;
+  if (record) {                                   // entries at their record order (STACK); the heads
+                                                  // are compacted straight into the record
     M.wit = o;  o += align256(max_entries);
     M.went = o; o += align256(4 * max_entries);
   }
@@ -503,8 +501,21 @@ __global__ void __launch_bounds__(kThreads) compact_kernel(const MCtl* ctl, cons
                                                            const uint32_t* __restrict__ stg_idx,
                                                            const uint32_t* __restrict__ stg_val,
                                                            float inv_div, int divide, uint32_t* __restrict__ out_idx,
-                                                           uint32_t* __restrict__ out_val) {
+                                                           uint32_t* __restrict__ out_val, uint8_t* __restrict__ rec,
+                                                           uint64_t rec_cap, uint32_t B, int stack) {
   const uint32_t num_items = ctl->num_items;
+  if (rec) {
+    // batch merge (round 2): the heads go straight to the record's idx and val/off sections, whose
+    // offsets are known once the unique count is (ucount_scan_kernel ran before); the packer then
+    // only writes the header, lr[], the padding, off[nnz] and the entry sections
+    const uint64_t nnz = ctl->nnz, nent = ctl->nent;
+    const uint64_t o_idx = 80 + pad16(4ull * B), o_v = o_idx + pad16(4 * nnz);
+    const uint64_t total = stack ? o_v + pad16(4 * (nnz + 1)) + pad16(nent) + pad16(4 * nent)
+                                 : o_v + pad16(4 * nnz);
+    if (total > rec_cap) return;                     // the packer reports the size; nothing is written
+    out_idx = reinterpret_cast<uint32_t*>(rec + o_idx);
+    out_val = reinterpret_cast<uint32_t*>(rec + o_v);
+  }
   const int lane = threadIdx.x & 31;
   (void)inv_div;
   for (uint32_t i = (blockIdx.x * kThreads + threadIdx.x) >> 5; i < num_items; i += (gridDim.x * kThreads) >> 5) {
@@ -606,8 +617,6 @@ struct PackArgs {
 };
 
 __global__ void __launch_bounds__(kThreads) pack_kernel(const __grid_constant__ PackArgs a, const MCtl* ctl,
-                                                        const uint32_t* __restrict__ widx,
-                                                        const uint32_t* __restrict__ wval,
                                                         const uint8_t* __restrict__ wit,
                                                         const uint32_t* __restrict__ went,
                                                         uint8_t* __restrict__ rec, uint64_t* d_bytes) {
@@ -623,10 +632,20 @@ __global__ void __launch_bounds__(kThreads) pack_kernel(const __grid_constant__ 
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) *d_bytes = total;
   if (total > a.cap) return;
+  const uint64_t o_heads_end = a.mode == LOWDIFF_MERGE_SUM ? total : o_it;   // idx + val/off: compact_kernel
+  if (blockIdx.x == 0 && threadIdx.x < 8) {        // their zero padding (whole words) and off[nnz] = nent
+    uint32_t* w32 = reinterpret_cast<uint32_t*>(rec);
+    const int t = threadIdx.x;
+    const uint64_t e_idx = o_idx + 4 * nnz, e_v = o_v + 4 * (a.mode == LOWDIFF_MERGE_SUM ? nnz : nnz + 1);
+    if (e_idx / 4 + t < o_v / 4 && t < 4) w32[e_idx / 4 + t] = 0u;
+    if (t >= 4 && e_v / 4 + (t - 4) < o_heads_end / 4) w32[e_v / 4 + (t - 4)] = 0u;
+    if (t == 0 && a.mode != LOWDIFF_MERGE_SUM) w32[o_v / 4 + nnz] = (uint32_t)nent;
+  }
   const uint64_t chunks = total / 16;
   for (uint64_t c = (uint64_t)blockIdx.x * kThreads + threadIdx.x; c < chunks;
        c += (uint64_t)gridDim.x * kThreads) {
     const uint64_t off = c * 16;
+    if (off >= o_idx && off < o_heads_end) continue;   // written by compact_kernel (+ the padding above)
     uint32_t wd[4];
     if (off < o_lr) {                          // header
 #pragma unroll
@@ -655,19 +674,6 @@ __global__ void __launch_bounds__(kThreads) pack_kernel(const __grid_constant__ 
       for (int q = 0; q < 4; ++q) {
         const uint64_t j = (off - o_lr) / 4 + q;
         wd[q] = j < a.B ? __float_as_uint(a.lr[j]) : 0u;
-      }
-    } else if (off < o_v) {                    // idx[nnz]
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const uint64_t j = (off - o_idx) / 4 + q;
-        wd[q] = j < nnz ? widx[j] : 0u;
-      }
-    } else if (a.mode == LOWDIFF_MERGE_SUM || off < o_it) {   // SUM val[nnz] / STACK off[nnz+1]
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const uint64_t j = (off - o_v) / 4 + q;
-        if (a.mode == LOWDIFF_MERGE_SUM) wd[q] = j < nnz ? wval[j] : 0u;
-        else wd[q] = j < nnz ? wval[j] : (j == nnz ? (uint32_t)nent : 0u);
       }
     } else if (off < o_ent) {                  // it[nent] (u8)
 #pragma unroll
@@ -814,11 +820,13 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
               ucnt, epre, sidx, sval, oit, oent, sparse_max, bitmap_min);
   LD_LAUNCH(cls, s, ucount_scan_kernel, 1, kPlanThreads, 0, ls, M.num_w, starts, ctl, ucnt, upre,
             kind == kCoalesce ? d_out_nnz : nullptr);
-  uint32_t* didx = record ? reinterpret_cast<uint32_t*>(w + M.widx) : out_idx;
-  uint32_t* dval = record ? reinterpret_cast<uint32_t*>(w + M.wval) : reinterpret_cast<uint32_t*>(out_val);
+  uint32_t* didx = record ? nullptr : out_idx;     // record: compact_kernel places the heads in it
+  uint32_t* dval = record ? nullptr : reinterpret_cast<uint32_t*>(out_val);
   const int cgrid = (int)((M.num_w + 7) / 8 < 4u * kNumSMs ? (M.num_w + 7) / 8 : 4u * kNumSMs);
   LD_LAUNCH(cls, s, compact_kernel, cgrid, kThreads, 0, ctl, ucnt, epre, upre, sidx, sval, (float)ls.L,
-            (kind == kCoalesce && average) ? 1 : 0, didx, dval);
+            (kind == kCoalesce && average) ? 1 : 0, didx, dval,
+            record ? static_cast<uint8_t*>(d_record) : nullptr, record ? record_cap : 0, (uint32_t)ls.L,
+            kind == kMergeStack ? 1 : 0);
   if (kind == kCoalesce) return cuda_status(cudaGetLastError(), "coalesce launch");
 
   PackArgs pa;
@@ -831,9 +839,7 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
   uint64_t pg = (est + kThreads - 1) / kThreads;
   if (pg > 8ull * kNumSMs) pg = 8ull * kNumSMs;
   if (pg < 1) pg = 1;
-  LD_LAUNCH("merge_pack", s, pack_kernel, (int)pg, kThreads, 0, pa, ctl,
-            reinterpret_cast<const uint32_t*>(w + M.widx), reinterpret_cast<const uint32_t*>(w + M.wval),
-            w + M.wit, reinterpret_cast<const uint32_t*>(w + M.went), static_cast<uint8_t*>(d_record),
+  LD_LAUNCH("merge_pack", s, pack_kernel, (int)pg, kThreads, 0, pa, ctl, w + M.wit, reinterpret_cast<const uint32_t*>(w + M.went), static_cast<uint8_t*>(d_record),
             d_record_bytes);
   return cuda_status(cudaGetLastError(), "merge launch");
 }
