@@ -397,24 +397,28 @@ def run_ours(args, cfg):
         """Batch merge -> record b -> async D2H stage (copy stream); returns the record's bytes."""
         diffs = [(ring[j][0], ring[j][1], ring[j][2], cap, lr) for j in range(B)]
         ld.batch_merge(diffs, cfg.merge, n, lo, hi, t_iter[0], P, record=records[b], d_record_bytes=d_bytes)
-        nb = ld.record_bytes(d_bytes, rec_cap)          # the checkpoint thread's only sync
         ld.stage_d2h(records[b], 80 + 4 * B, heads[b], main)   # header + lr[] for the host-side replay
-        copy_stream.wait_stream(main)
-        ld.stage_d2h(records[b], nb, staged[b], copy_stream)   # async persist staging (copy engine)
+        nb = ld.record_bytes(d_bytes, rec_cap)          # the checkpoint thread's only sync (covers the header)
         rec_nb[b] = nb
         t_iter[0] += B
-        return nb
+        if b < R - 1:                                   # the last record is staged behind the replay launch
+            ld.stage_d2h(records[b], nb, staged[b], copy_stream)   # async persist staging (copy engine);
+        return nb                                       # the record is complete: the host just synced
 
     def recovery_phase():
-        """Load(C^F) + replay of the step's chain of R records (K = R*B iterations)."""
-        main.synchronize()                              # the replay call reads the staged headers
+        """Load(C^F) + replay of the step's chain of R records (K = R*B iterations); the headers were
+        copied before the last record_bytes synchronization, so the replay launches at once and the
+        last record's staging is issued right after it (the copy engine works beside the replay)."""
         if os.environ.get("LOWDIFF_BENCH_SERIAL_STAGE"):  # experiment: staging not overlapped with replay
+            ld.stage_d2h(records[R - 1], rec_nb[R - 1], staged[R - 1], copy_stream)
             copy_stream.synchronize()
         state["t"] = t_iter[0] - R * B                  # the checkpoint is stamped at the chain start
         state["adam_step"] = ck["adam_step"]
         state["momentum_initialized"] = ck["momentum_initialized"]
         ld.replay(state, opt, [(records[b], heads[b]) for b in range(R)], check=False)
-        main.wait_stream(copy_stream)
+        if not os.environ.get("LOWDIFF_BENCH_SERIAL_STAGE"):
+            ld.stage_d2h(records[R - 1], rec_nb[R - 1], staged[R - 1], copy_stream)
+        main.wait_stream(copy_stream)                   # the next step's merge overwrites the records
 
     def step(graph=None, h2d=None):
         """One pass of the path: R batches built, merged and staged, then the chain replayed."""
