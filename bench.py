@@ -555,8 +555,8 @@ def run_ours(args, cfg):
         if cfg.opt == "adam" and opt.get("approx_math"):
             # approx_math: one MUFU.RSQ and 6 fp32 lane-ops (FFMA2/FMUL2 pairs) per
             # parameter-step in the zero-gradient steps; the XU pipe issues 16 lanes/clk/SM (ncu: the
-            # two-MUFU form ran XU-bound at 79 % of it) and the fp32 pipe 128 lanes/clk/SM, so both
-            # give 16 parameter-steps/clk/SM: that is the floor.
+            # two-MUFU form ran XU-bound at 79 % of it) and the fp32 pipe 128 lanes/clk/SM (21
+            # parameter-steps/clk/SM), so the XU's 16 parameter-steps/clk/SM is the floor.
             f_mhz = (clk or {}).get("sm_mhz") or 1965.0
             psteps = nloc * R * B
             floor_s = psteps / (148 * 16 * f_mhz * 1e6)
