@@ -63,7 +63,8 @@ for mode in ("sum", "stack"):
 x0 = torch.randn(n, device=dev) * 0.05
 for kind, opt, rr in (("sgd", {"kind": "sgd"}, recs[0]), ("sgd", {"kind": "sgd", "weight_decay": 1e-4}, recs[1]),
                       ("momentum", {"kind": "momentum", "momentum": 0.9, "dampening": 0.1}, recs[1]),
-                      ("adam", {"kind": "adam", "beta1": 0.9, "beta2": 0.999, "eps": 1e-8}, recs[1])):
+                      ("adam", {"kind": "adam", "beta1": 0.9, "beta2": 0.999, "eps": 1e-8}, recs[1]),
+                      ("adam", {"kind": "adam", "beta1": 0.9, "beta2": 0.999, "eps": 1e-8, "approx_math": 1}, recs[1])):
     st = {"x": x0.clone(), "m": None if kind == "sgd" else torch.zeros(n, device=dev),
           "v": torch.full((n,), 1e-8, device=dev) if kind == "adam" else None,
           "x_bf16": torch.empty(n, dtype=torch.bfloat16, device=dev) if kind == "adam" else None,
