@@ -314,7 +314,8 @@ typedef struct {
                                          oracle. 1: the step's sqrt and division as single MUFU ops
                                          (sqrt.approx, rcp.approx): m, v as in 0, x within north_star's
                                          fp32 tolerance (1e-6 rel / 1e-7 abs) of the oracle, x_bf16 within
-                                         2^-7 rel; no range gate (reading #33). */
+                                         2^-7 rel; no range gate (reading #33). Honoured for
+                                         eps >= 2^-40; with a smaller eps the mode-0 kernel runs. */
 } lowdiff_opt;
 
 typedef struct {
