@@ -151,12 +151,13 @@ struct SparseSmem {
 };
 constexpr int kBmLists = 32;                // lists the bitmap path handles
 constexpr int kWords = kW / 32;             // bitmap words per fine window
-constexpr int kBmWords = 6144;              // list x word capacity of a bitmap item (24 KB)
-constexpr int kBmMaxWords = 768;            // words (6 windows) per bitmap item
+constexpr int kBmWords = 4096;              // list x word capacity of a bitmap item (16 KB)
+constexpr int kBmMaxWords = 512;            // words (4 windows) per bitmap item
 struct BitmapSmem {
   uint32_t bm[kBmWords];           // per list, the item's occupied slots (list-major)
   uint64_t wpre[kBmMaxWords];      // per word: (# unique slots before it) << 32 | # entries before it
-  uint32_t orw[kBmMaxWords];       // per word: slots occupied by any list
+  uint4 pl[kBmMaxWords];           // per word, L <= 15: bit planes of the per-slot list count
+                                   // (x = 1s, y = 2s, z = 4s, w = 8s); L > 15: x = slots of any list
 };
 union ItemSmem {
   DenseSmem d;
@@ -244,25 +245,57 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
           if (sl[u] != 0xFFFFFFFFu) atomicOr(&sm.b.bm[aa[u] * NW + (sl[u] >> 5)], 1u << (sl[u] & 31));
       }
       __syncthreads();
-      // each thread owns q consecutive words: their counts, a block scan, then the per-word prefix
+      // each thread owns q consecutive words: their counts, a block scan, then the per-word prefix.
+      // Up to 15 lists the word's per-slot list counts are kept as 4 bit planes (a carry-save sum of
+      // the lists' bitmaps), so an entry's count of entries at lower slots of its word is 4
+      // popcounts instead of a loop over the lists, and only a slot held by >= 2 lists walks the
+      // lists for its iteration rank (round 2; C4: ~2 % of the slots)
+      const bool planes = L <= 15;
+      constexpr int kQ = (kBmMaxWords + kThreads - 1) / kThreads;
       const uint32_t q = (NW + kThreads - 1) / kThreads, w_a = tid * q, w_e = min(NW, w_a + q);
+      uint64_t cw[kQ];
       uint64_t mine = 0;
-      for (uint32_t wd = w_a; wd < w_e; ++wd) {
-        uint32_t orv = 0, c = 0;
-        for (int l = 0; l < L; ++l) {
-          const uint32_t bw = sm.b.bm[l * NW + wd];
-          orv |= bw;
-          c += __popc(bw);
+#pragma unroll
+      for (int i = 0; i < kQ; ++i) {
+        const uint32_t wd = w_a + i;
+        cw[i] = 0;
+        if (wd >= w_e) continue;
+        uint32_t c, u;
+        if (planes) {
+          uint32_t p0 = 0, p1 = 0, p2 = 0, p3 = 0;
+          for (int l = 0; l < L; ++l) {
+            const uint32_t b = sm.b.bm[l * NW + wd];
+            const uint32_t c0 = p0 & b;
+            p0 ^= b;
+            const uint32_t c1 = p1 & c0;
+            p1 ^= c0;
+            const uint32_t c2 = p2 & c1;
+            p2 ^= c1;
+            p3 ^= c2;
+          }
+          sm.b.pl[wd] = make_uint4(p0, p1, p2, p3);
+          c = __popc(p0) + 2 * __popc(p1) + 4 * __popc(p2) + 8 * __popc(p3);
+          u = __popc(p0 | p1 | p2 | p3);
+        } else {
+          uint32_t orv = 0;
+          c = 0;
+          for (int l = 0; l < L; ++l) {
+            const uint32_t bw = sm.b.bm[l * NW + wd];
+            orv |= bw;
+            c += __popc(bw);
+          }
+          sm.b.pl[wd].x = orv;
+          u = __popc(orv);
         }
-        sm.b.orw[wd] = orv;
-        mine += ((uint64_t)__popc(orv) << 32) | c;
+        cw[i] = ((uint64_t)u << 32) | c;
+        mine += cw[i];
       }
       uint64_t run = block_exclusive_scan(mine, s_scan, &tot);
-      for (uint32_t wd = w_a; wd < w_e; ++wd) {
-        sm.b.wpre[wd] = run;
-        uint32_t c = 0;
-        for (int l = 0; l < L; ++l) c += __popc(sm.b.bm[l * NW + wd]);
-        run += ((uint64_t)__popc(sm.b.orw[wd]) << 32) | c;
+#pragma unroll
+      for (int i = 0; i < kQ; ++i) {
+        if (w_a + i >= w_e) continue;
+        sm.b.wpre[w_a + i] = run;
+        run += cw[i];
       }
       __syncthreads();
       for (uint32_t x0 = tid; x0 < E; x0 += 4 * kThreads) {   // 4 entries' (idx, val) loads in flight
@@ -283,18 +316,27 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
         const int a = aa[u];
         const uint32_t slot = sl[u];
         const uint32_t wd = slot >> 5, bit = 1u << (slot & 31), below = bit - 1u;
-        uint32_t cb = 0, rank = 0;
-        for (int l = 0; l < L; ++l) {
-          const uint32_t bw = sm.b.bm[l * NW + wd];
-          cb += __popc(bw & below);
-          rank += (l < a && (bw & bit)) ? 1u : 0u;
+        uint32_t cb = 0, rank = 0, orw;
+        if (planes) {
+          const uint4 P = sm.b.pl[wd];
+          cb = __popc(P.x & below) + 2 * __popc(P.y & below) + 4 * __popc(P.z & below) + 8 * __popc(P.w & below);
+          orw = P.x | P.y | P.z | P.w;
+          if ((P.y | P.z | P.w) & bit)             // a slot of >= 2 lists: its lists before this one
+            for (int l = 0; l < a; ++l) rank += (sm.b.bm[l * NW + wd] & bit) ? 1u : 0u;
+        } else {
+          for (int l = 0; l < L; ++l) {
+            const uint32_t bw = sm.b.bm[l * NW + wd];
+            cb += __popc(bw & below);
+            rank += (l < a && (bw & bit)) ? 1u : 0u;
+          }
+          orw = sm.b.pl[wd].x;
         }
         const uint64_t pw = sm.b.wpre[wd];
         const uint32_t pos = e0 + (uint32_t)pw + cb + rank;
         out_it[pos] = (uint8_t)a;
         out_ent[pos] = vv[u];
         if (rank == 0) {
-          const uint32_t uu = e0 + (uint32_t)(pw >> 32) + __popc(sm.b.orw[wd] & below);
+          const uint32_t uu = e0 + (uint32_t)(pw >> 32) + __popc(orw & below);
           stg_idx[uu] = (uint32_t)(w0 + slot);
           stg_val[uu] = pos;                       // off[] = the head's entry position
         }
