@@ -166,7 +166,7 @@ union ItemSmem {
 };
 
 template <int KIND, bool BF16>
-__global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__ ListSet ls, uint64_t lo,
+__global__ void __launch_bounds__(kThreads, 6) merge_kernel(const __grid_constant__ ListSet ls, uint64_t lo,
                                                          uint32_t num_w, const uint32_t* __restrict__ starts,
                                                          const uint2* __restrict__ items, MCtl* ctl,
                                                          uint32_t* __restrict__ ucnt, uint32_t* __restrict__ epre,
@@ -231,18 +231,20 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
       //      and the first entry of a slot (rank 0) writes the unique head. No sorting.
       for (uint32_t j = tid; j < (uint32_t)L * NW; j += kThreads) sm.b.bm[j] = 0;
       __syncthreads();
-      for (uint32_t x0 = tid; x0 < E; x0 += 4 * kThreads) {   // 4 entries' loads in flight
-        int aa[4];
-        uint32_t sl[4];
+      // warp w walks lists w, w + 8, ... (no per-entry list lookup; round 2: the binary search over
+      // the lists' offsets was ~20 % of the kernel's issue slots), 4 entries per lane in flight
+      const int bw_warp = tid >> 5, bw_lane = tid & 31;
+      for (int l = bw_warp; l < L; l += kThreads / 32) {
+        const uint32_t* li = ls.list[l].idx + s_beg[l];
+        const uint32_t len = s_len[l];
+        for (uint32_t j0 = bw_lane; j0 < len; j0 += 128) {
+          uint32_t sl[4];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const uint32_t x = x0 + u * kThreads;
-          aa[u] = x < E ? list_of(x) : 0;
-          sl[u] = x < E ? ls.list[aa[u]].idx[s_beg[aa[u]] + (x - s_off[aa[u]])] - (uint32_t)w0 : 0xFFFFFFFFu;
+          for (int u = 0; u < 4; ++u) sl[u] = j0 + 32 * u < len ? li[j0 + 32 * u] - (uint32_t)w0 : 0xFFFFFFFFu;
+#pragma unroll
+          for (int u = 0; u < 4; ++u)
+            if (sl[u] != 0xFFFFFFFFu) atomicOr(&sm.b.bm[l * NW + (sl[u] >> 5)], 1u << (sl[u] & 31));
         }
-#pragma unroll
-        for (int u = 0; u < 4; ++u)
-          if (sl[u] != 0xFFFFFFFFu) atomicOr(&sm.b.bm[aa[u] * NW + (sl[u] >> 5)], 1u << (sl[u] & 31));
       }
       __syncthreads();
       // each thread owns q consecutive words: their counts, a block scan, then the per-word prefix.
@@ -298,22 +300,22 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
         run += cw[i];
       }
       __syncthreads();
-      for (uint32_t x0 = tid; x0 < E; x0 += 4 * kThreads) {   // 4 entries' (idx, val) loads in flight
-        int aa[4];
+      for (int a = bw_warp; a < L; a += kThreads / 32) {   // the same walk: list a's entries
+        const uint64_t eb = s_beg[a];
+        const uint32_t* li = ls.list[a].idx + eb;
+        const uint32_t len = s_len[a];
+        for (uint32_t j0 = bw_lane; j0 < len; j0 += 128) {   // 4 entries' (idx, val) loads in flight
         uint32_t sl[4];
         float vv[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
-          const uint32_t x = x0 + u * kThreads;
-          aa[u] = x < E ? list_of(x) : 0;
-          const uint64_t e = s_beg[aa[u]] + (x - s_off[aa[u]]);
-          sl[u] = x < E ? ls.list[aa[u]].idx[e] - (uint32_t)w0 : 0xFFFFFFFFu;
-          vv[u] = x < E ? list_val<BF16>(ls, aa[u], e) : 0.f;
+          const uint32_t e = j0 + 32 * u;
+          sl[u] = e < len ? li[e] - (uint32_t)w0 : 0xFFFFFFFFu;
+          vv[u] = e < len ? list_val<BF16>(ls, a, eb + e) : 0.f;
         }
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
         if (sl[u] == 0xFFFFFFFFu) break;
-        const int a = aa[u];
         const uint32_t slot = sl[u];
         const uint32_t wd = slot >> 5, bit = 1u << (slot & 31), below = bit - 1u;
         uint32_t cb = 0, rank = 0, orw;
@@ -339,6 +341,7 @@ __global__ void __launch_bounds__(kThreads) merge_kernel(const __grid_constant__
           const uint32_t uu = e0 + (uint32_t)(pw >> 32) + __popc(orw & below);
           stg_idx[uu] = (uint32_t)(w0 + slot);
           stg_val[uu] = pos;                       // off[] = the head's entry position
+        }
         }
         }
       }
