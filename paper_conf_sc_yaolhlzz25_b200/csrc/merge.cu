@@ -828,7 +828,9 @@ lowdiff_status merge_run(const ListSet& ls, MergeKind kind, uint64_t lo, uint64_
   const uint32_t merge_ctas = 6u * kNumSMs;
   if (kind == kMergeStack && ls.L <= 16 && per_w >= (double)bitmap_min) {
     G = 1;                          // groups of bitmap size: as many windows as fit (power of 2)
-    while (2 * G * kWords <= (uint32_t)kBmMaxWords && (uint32_t)ls.L * 2 * G * kWords <= (uint32_t)kBmWords &&
+    uint32_t gmax = 1u << 30;                       // experiments: LOWDIFF_MERGE_BMG caps the windows per item
+    if (const char* e = getenv("LOWDIFF_MERGE_BMG")) gmax = (uint32_t)atoi(e);
+    while (2 * G <= gmax && 2 * G * kWords <= (uint32_t)kBmMaxWords && (uint32_t)ls.L * 2 * G * kWords <= (uint32_t)kBmWords &&
            M.num_w / (2 * G) >= 4 * merge_ctas)
       G <<= 1;
     keep_groups = 1;
