@@ -165,8 +165,11 @@ union ItemSmem {
   BitmapSmem b;
 };
 
+#ifndef LOWDIFF_MERGE_MINB
+#define LOWDIFF_MERGE_MINB 6                    // CTAs per SM the item engine is compiled for (37 KB smem each)
+#endif
 template <int KIND, bool BF16>
-__global__ void __launch_bounds__(kThreads, 6) merge_kernel(const __grid_constant__ ListSet ls, uint64_t lo,
+__global__ void __launch_bounds__(kThreads, LOWDIFF_MERGE_MINB) merge_kernel(const __grid_constant__ ListSet ls, uint64_t lo,
                                                          uint32_t num_w, const uint32_t* __restrict__ starts,
                                                          const uint2* __restrict__ items, MCtl* ctl,
                                                          uint32_t* __restrict__ ucnt, uint32_t* __restrict__ epre,
