@@ -342,7 +342,9 @@ def run_ours(args, cfg):
     rec_cap = ld.record_max_bytes(cfg.merge, B, B * cap, lo, hi)
     R = chain_records(cfg)                              # batch records per step (replay chain K = R*B)
     records = [torch.empty(rec_cap, dtype=torch.uint8, device=dev) for _ in range(R)]
-    d_bytes = torch.zeros(1, dtype=torch.int64, device=dev)
+    d_bytes = [torch.zeros(1, dtype=torch.int64, device=dev) for _ in range(R)]   # one per record
+    meta = torch.cuda.Stream(device=dev)             # the checkpoint thread's size queries
+    rec_done = [torch.cuda.Event() for _ in range(R)]
     heads = [torch.empty(80 + 4 * B + 16, dtype=torch.uint8, pin_memory=True) for _ in range(R)]
     staged = [torch.empty(rec_cap, dtype=torch.uint8, pin_memory=True) for _ in range(R)]
     main = torch.cuda.current_stream()
@@ -394,13 +396,20 @@ def run_ours(args, cfg):
     rec_nb = [0] * R
 
     def checkpoint_phase(b):
-        """Batch merge -> record b -> async D2H stage (copy stream); returns the record's bytes."""
+        """Batch merge -> record b (+ its header D2H for the host-side replay), enqueued on the
+        training stream; the size query and the staging follow in finish(b)."""
         diffs = [(ring[j][0], ring[j][1], ring[j][2], cap, lr) for j in range(B)]
-        ld.batch_merge(diffs, cfg.merge, n, lo, hi, t_iter[0], P, record=records[b], d_record_bytes=d_bytes)
+        ld.batch_merge(diffs, cfg.merge, n, lo, hi, t_iter[0], P, record=records[b], d_record_bytes=d_bytes[b])
         ld.stage_d2h(records[b], 80 + 4 * B, heads[b], main)   # header + lr[] for the host-side replay
-        nb = ld.record_bytes(d_bytes, rec_cap)          # the checkpoint thread's only sync (covers the header)
-        rec_nb[b] = nb
+        rec_done[b].record(main)
         t_iter[0] += B
+
+    def finish(b):
+        """The checkpoint thread learns record b's size on its own stream (waits for record b only:
+        the training stream has already moved on to the next batch's compress), then stages it."""
+        meta.wait_event(rec_done[b])
+        nb = ld.record_bytes(d_bytes[b], rec_cap, stream=meta)   # syncs `meta` (covers the header)
+        rec_nb[b] = nb
         if b < R - 1:                                   # the last record is staged behind the replay launch
             ld.stage_d2h(records[b], nb, staged[b], copy_stream)   # async persist staging (copy engine);
         return nb                                       # the record is complete: the host just synced
@@ -428,7 +437,10 @@ def run_ours(args, cfg):
                 graph.replay()
             else:
                 build_phase(h2d)
-            nb += checkpoint_phase(b)
+            checkpoint_phase(b)
+            if b:
+                nb += finish(b - 1)                     # record b-1's size while batch b builds
+        nb += finish(R - 1)
         recovery_phase()
         return nb
 
