@@ -565,17 +565,17 @@ def run_ours(args, cfg):
                        "achieved_gbs": alg / t_s / 1e9, "hbm_frac": alg / t_s / 1e9 / hbm_peak,
                        "ms_per_step": rp_ms / args.steps}
         if cfg.opt == "adam" and opt.get("approx_math"):
-            # approx_math: one MUFU.RSQ and 6 fp32 lane-ops (FFMA2/FMUL2 pairs) per
-            # parameter-step in the zero-gradient steps; the XU pipe issues 16 lanes/clk/SM (ncu: the
-            # two-MUFU form ran XU-bound at 79 % of it) and the fp32 pipe 128 lanes/clk/SM (21
-            # parameter-steps/clk/SM), so the XU's 16 parameter-steps/clk/SM is the floor.
+            # approx_math: in the zero-gradient loop one MUFU.RSQ every other step
+            # (0.5 per parameter-step; the XU pipe issues 16 lanes/clk/SM: 32 parameter-steps/clk/SM)
+            # and 6.5 fp32 lane-ops per parameter-step (FFMA2/FMUL2; 128 lanes/clk/SM: 19.7
+            # parameter-steps/clk/SM): the fp32 pipe is the floor.
             f_mhz = (clk or {}).get("sm_mhz") or 1965.0
             psteps = nloc * R * B
-            floor_s = psteps / (148 * 16 * f_mhz * 1e6)
+            floor_s = psteps / (148 * (128 / 6.5) * f_mhz * 1e6)
             replay_roof.update({"bound": "alu", "math": "approx", "alu_floor_ms": floor_s * 1e3,
                                 "alu_frac": floor_s / t_s,
-                                "alu_peak": f"16 parameter-steps/clk/SM x 148 SMs at {f_mhz:.0f} MHz (1 MUFU at "
-                                            "16 lanes/clk/SM; 6 fp32 lane-ops at 128 lanes/clk/SM)",
+                                "alu_peak": f"19.7 parameter-steps/clk/SM x 148 SMs at {f_mhz:.0f} MHz (6.5 fp32 "
+                                            "lane-ops at 128 lanes/clk/SM; 0.5 MUFU at 16 lanes/clk/SM)",
                                 "param_steps_per_s": psteps / t_s})
         elif cfg.opt == "adam":
             # Per parameter-step the exact Adam step issues 15 fp32 operations (FFMA2 pairs) and 2
