@@ -311,8 +311,9 @@ typedef struct {
   int32_t nesterov;
   int32_t allow_accumulated_sum;
   int32_t approx_math;                /* Adam only. 0: every op correctly rounded, x/m/v bit-exact vs the
-                                         oracle. 1: the step's sqrt and division as single MUFU ops
-                                         (sqrt.approx, rcp.approx): m, v as in 0, x within north_star's
+                                         oracle. 1: the step's sqrt and division through MUFU approximations
+                                         (rsqrt and a short series for 1/(1 + eps/sqrt(v)); sqrt.approx and
+                                         rcp.approx where the series does not apply): m, v as in 0, x within north_star's
                                          fp32 tolerance (1e-6 rel / 1e-7 abs) of the oracle, x_bf16 within
                                          2^-7 rel; no range gate (reading #33). Honoured for
                                          eps >= 2^-40; with a smaller eps the mode-0 kernel runs. */
