@@ -214,10 +214,41 @@ def run_reference(args, cfg):
 # GPU arm
 # ---------------------------------------------------------------------------------------------
 class ClockSampler:
+    """SM clock and clock-event (throttle) reasons DURING the timed region: NVML polled every ~5 ms
+    from a thread (one sample at start() and one at stop() as well, so even a few-millisecond timed
+    region has samples); nvidia-smi -lms 20 only if NVML is unavailable."""
+
     def __init__(self, index: int):
-        self.index, self.proc, self.path = index, None, None
+        self.index, self.proc, self.path, self.thread = index, None, None, None
+        self.samples, self.stop_flag = [], False
+
+    def _nvml_sample(self):
+        import pynvml
+        sm = pynvml.nvmlDeviceGetClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        mx = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        try:
+            bits = pynvml.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+        except Exception:
+            bits = pynvml.nvmlDeviceGetCurrentClocksThrottleReasons(self.h)
+        self.samples.append((float(sm), float(mx), int(bits)))
 
     def start(self):
+        try:
+            import threading
+            import pynvml
+            pynvml.nvmlInit()
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            self._nvml_sample()
+
+            def run():
+                while not self.stop_flag:
+                    self._nvml_sample()
+                    time.sleep(0.005)
+            self.thread = threading.Thread(target=run, daemon=True)
+            self.thread.start()
+            return
+        except Exception:
+            self.thread = None
         try:
             self.path = os.path.join("/tmp", f"lowdiff_clocks_{os.getpid()}.csv")
             self.f = open(self.path, "w")
@@ -229,31 +260,33 @@ class ClockSampler:
             self.proc = None
 
     def stop(self):
-        if self.proc is None:
-            return None
-        self.proc.terminate()
-        try:
-            self.proc.wait(timeout=5)
-        except Exception:
-            self.proc.kill()
-        self.f.close()
-        sm, mx, reasons = [], 0.0, set()
-        for line in open(self.path):
-            parts = [p.strip() for p in line.split(",")]
-            if len(parts) < 3:
-                continue
+        if self.thread is not None:
+            self.stop_flag = True
+            self.thread.join()
+            self._nvml_sample()
+            rows = self.samples
+        elif self.proc is not None:
+            self.proc.terminate()
             try:
-                sm.append(float(parts[0])); mx = max(mx, float(parts[1]))
-                bits = int(parts[2], 16)
-                for b, name in REASONS.items():
-                    if bits & b and name != "gpu_idle":
-                        reasons.add(name)
-            except ValueError:
-                continue
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+            self.f.close()
+            rows = []
+            for line in open(self.path):
+                parts = [p.strip() for p in line.split(",")]
+                try:
+                    rows.append((float(parts[0]), float(parts[1]), int(parts[2], 16)))
+                except (ValueError, IndexError):
+                    continue
+        else:
+            return None
+        sm = [r[0] for r in rows]
         if not sm:
             return None
-        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
-                "samples": len(sm)}
+        reasons = {name for r in rows for b, name in REASONS.items() if r[2] & b and name != "gpu_idle"}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(r[1] for r in rows),
+                "reasons": sorted(reasons), "samples": len(sm)}
 
 
 def run_ours(args, cfg):
