@@ -207,7 +207,7 @@ def run_reference(args, cfg):
             "cpu_baseline": {"value": val, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample,
                              **host_description()},
             "e2e": {"value": val, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(line), flush=True)
+    emit(line)
 
 
 # ---------------------------------------------------------------------------------------------
@@ -785,7 +785,7 @@ def run_ours(args, cfg):
                            "profiled": "separate pass, eager launches, CUDA events around every kernel"},
                 "roofline": roofline, "replay_roofline": replay_roof, "replay_math": replay_exact, "stage": stage, "kernels": kernels, "cpu_baseline": cpu, "e2e": e2e,
                 "gpu_launches": int(launches), "clocks": clk}
-        print(json.dumps(line), flush=True)
+        emit(line)
     if comm is not None:
         comm.destroy()
     if p2p is not None:
@@ -795,7 +795,27 @@ def run_ours(args, cfg):
         dist.destroy_process_group()
 
 
+_JSON_OUT = None                                     # the real stdout when it is redirected (N > 1)
+
+
+def emit(line: dict):
+    """The one JSON line of this run, on the process's real stdout."""
+    if _JSON_OUT is not None:
+        _JSON_OUT.write(json.dumps(line) + "\n")
+        _JSON_OUT.flush()
+    else:
+        print(json.dumps(line), flush=True)
+
+
 def main():
+    global _JSON_OUT
+    if int(os.environ.get("WORLD_SIZE", "1")) > 1:
+        # under torchrun, NCCL / c10d print banners (e.g. "NCCL version ...") on stdout at
+        # communicator creation: route fd 1 to stderr for the run and keep the real stdout for the
+        # JSON line alone
+        sys.stdout.flush()
+        _JSON_OUT = os.fdopen(os.dup(1), "w")
+        os.dup2(2, 1)
     args = parse_args()
     from workloads import CONFIGS
     cfg = CONFIGS[args.config]
