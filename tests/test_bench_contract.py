@@ -35,3 +35,15 @@ def test_reference_arm_nonzero_rank_is_silent():
     out = run(["--impl", "reference", "--config", "1", "--steps", "1", "--warmup", "0"], env={"RANK": "1"})
     assert out.returncode == 0
     assert out.stdout.strip() == ""
+
+
+def test_reference_arm_under_torchrun_env_prints_only_json():
+    """WORLD_SIZE > 1 (torchrun): fd 1 is routed to stderr for library banners (NCCL / c10d print
+    e.g. "NCCL version ..." on stdout) and the real stdout carries the one JSON line of rank 0."""
+    out = run(["--impl", "reference", "--config", "1", "--steps", "1", "--warmup", "0"],
+              env={"RANK": "0", "WORLD_SIZE": "2", "LOCAL_RANK": "0"})
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [ln for ln in out.stdout.splitlines() if ln.strip()]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["value"] > 0
